@@ -1,0 +1,164 @@
+/*
+ * airtopk.h — C ABI of the B200-native AIR Top-K library (libairtopk.so).
+ *
+ * AIR Top-K = Adaptive and Iteration-fused Radix Top-K, Zhang, Li, Naruse, Wang, SC'23
+ * (/root/reference/PAPER.md; "P:n" below = line n of that file).
+ *
+ * Operation (§2.1 "Problem Statement"): for each row L of `len` elements and
+ * K = k in [1, len], produce a value list V and an index list I of length K with
+ * L[I[i]] = V[i] and V[i] <= L[j] for every j not in I — the K smallest elements
+ * ("without loss of generality") or, with select_min = 0, the K largest.
+ * Batches of rows with the same len and K are solved together (§5.1).
+ *
+ * Method (all on the GPU, the host only enqueues kernels — P:50):
+ *   multi-pass MSD radix select over order-preserving key bits with b = 11-bit digits
+ *   (§2.3): per pass a histogram, an inclusive prefix sum, the target digit j
+ *   with psum[j-1] < K <= psum[j], and a filter that emits definite winners and keeps the
+ *   candidates; filter(i-1) and histogram(i) fused in one kernel (§3.1); the scan run by
+ *   the last CTA to finish; candidates buffered only while C < N/alpha, else the next pass
+ *   re-reads the input (§3.2, alpha = 128 as in P:210); early stop when K == C (§3.3).
+ *
+ * Semantics fixed by this library where the paper is silent:
+ *   - Order: IEEE-754 total order of the key bits (-NaN < -inf < ... < -0 < +0 < ... < +inf < +NaN);
+ *     u32 keys use their natural order. No floating-point arithmetic is performed on keys.
+ *   - Ties at the K-th key are broken by LOWEST index (row-local index; for
+ *     airtopk_select_with_idx, by the smallest in_idx VALUE).
+ *   - out_vals are raw bit copies of the selected input elements (NaN payloads, -0.0 preserved).
+ *   - The order of the K results within a row is UNSPECIFIED.
+ *
+ * Layout: keys are row-major [batch][len], contiguous, in DEVICE memory (any alignment of the
+ * element type). out_vals is [batch][k] of the key type, out_idx is [batch][k] int64, both device
+ * memory, row-local indices in [0, len). Outputs must not alias keys or the workspace.
+ *
+ * Ownership: the caller owns every buffer. The library never frees, retains or writes through
+ * caller pointers other than out_vals / out_idx / workspace, and never modifies keys.
+ * Calls are stateless and re-entrant: concurrent calls on different streams must use distinct
+ * workspaces (the convenience entry points allocate their own with cudaMallocAsync).
+ *
+ * Asynchrony / errors: every entry point except airtopk_select_host only ENQUEUES work on
+ * `stream` (no host synchronisation, no device->host copy) and returns:
+ *   AIRTOPK_OK         work enqueued;
+ *   AIRTOPK_EINVAL     null pointer, batch < 1, len < 1, k < 1 or k > len (K in [1, N]);
+ *   AIRTOPK_EDTYPE     unknown dtype;
+ *   AIRTOPK_ENOSPACE   workspace smaller than airtopk_workspace_bytes(...);
+ *   AIRTOPK_ECUDA      a CUDA launch/allocation failed (airtopk_last_cuda_error() has the code).
+ * Faults inside kernels surface at the caller's next synchronisation, as with any CUDA library.
+ * Nothing is written to the outputs when a status other than AIRTOPK_OK is returned.
+ */
+#ifndef AIRTOPK_H_
+#define AIRTOPK_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* cudaStream_t without requiring cuda_runtime.h; 0 = the legacy default stream. */
+typedef struct CUstream_st* airtopk_stream_t;
+
+typedef enum {
+  AIRTOPK_OK = 0,
+  AIRTOPK_EINVAL = 1,
+  AIRTOPK_EDTYPE = 2,
+  AIRTOPK_ENOSPACE = 3,
+  AIRTOPK_ECUDA = 4
+} airtopk_status;
+
+typedef enum {
+  AIRTOPK_F32 = 0,  /* IEEE binary32, r = 32 bits: 3 radix passes of 11/11/10 bits */
+  AIRTOPK_F16 = 1,  /* IEEE binary16, r = 16: 2 passes (11/5) */
+  AIRTOPK_BF16 = 2, /* bfloat16, r = 16: 2 passes */
+  AIRTOPK_F64 = 3,  /* IEEE binary64, r = 64: 6 passes (5 x 11 + 9) */
+  AIRTOPK_U32 = 4   /* unsigned 32-bit integers, natural order */
+} airtopk_dtype;
+
+/* Engine selection (airtopk_options.engine). */
+typedef enum {
+  AIRTOPK_ENGINE_AUTO = 0,
+  AIRTOPK_ENGINE_GRID = 1,    /* multi-CTA per row, one launch per pass, last-CTA scan */
+  AIRTOPK_ENGINE_CLUSTER = 2  /* one thread-block cluster per row, all passes in one launch */
+} airtopk_engine;
+
+/* Tuning / ablation knobs. Pass NULL for the defaults. */
+typedef struct {
+  int64_t alpha;        /* adaptive-buffer parameter: buffer candidates iff C * alpha < len.
+                           0 = default 128; alpha >= len = never buffer; 1 = buffer
+                           whenever at least one element was eliminated. Must be >= 0. */
+  int32_t engine;       /* airtopk_engine; 0 = auto */
+  int32_t ctas_per_row; /* grid engine: CTAs per row; 0 = auto (fills the 148 SMs) */
+  int32_t cluster_size; /* cluster engine: CTAs per cluster (1,2,4,8,16); 0 = auto */
+  int32_t n_events;     /* number of entries in `events` */
+  int64_t* trace;       /* optional DEVICE buffer of batch * AIRTOPK_TRACE_MAX_PASSES * 10 int64:
+                           per-row state after each scan (width, src_is_input, stored, j, K, C, C',
+                           emitted_so_far, early_stop, elements_read); unused slots untouched.
+                           Grid engine only. NULL = no trace. */
+  void* const* events;  /* optional array of n_events cudaEvent_t (created by the caller) recorded on
+                           `stream` around the launches: events[0] before the first kernel,
+                           events[q+1] after launch q — lets a caller time each kernel with CUDA
+                           events on the launching stream. NULL = none. */
+} airtopk_options;
+
+#define AIRTOPK_TRACE_MAX_PASSES 16
+
+/* Bytes of device workspace a call with these arguments needs (grows with batch * len / alpha:
+ * two candidate buffers of floor((len-1)/alpha) entries per row). 0 on invalid arguments. */
+size_t airtopk_workspace_bytes(airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k);
+size_t airtopk_workspace_bytes_ex(airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k,
+                                  const airtopk_options* opt);
+
+/* Generic entry point. workspace: device memory of at least airtopk_workspace_bytes_ex(...) bytes,
+ * 256-byte aligned, owned by the caller, not used concurrently by another call. */
+airtopk_status airtopk_select(const void* keys, airtopk_dtype dtype, int64_t batch, int64_t len,
+                              int64_t k, int select_min, void* out_vals, int64_t* out_idx,
+                              void* workspace, size_t workspace_bytes, airtopk_stream_t stream);
+airtopk_status airtopk_select_ex(const void* keys, airtopk_dtype dtype, int64_t batch, int64_t len,
+                                 int64_t k, int select_min, void* out_vals, int64_t* out_idx,
+                                 void* workspace, size_t workspace_bytes, airtopk_stream_t stream,
+                                 const airtopk_options* opt);
+
+/* north_star signature, one per dtype: the workspace is taken from the stream-ordered pool
+ * (cudaMallocAsync / cudaFreeAsync on `stream`), so these are also fully asynchronous.
+ * 16-bit keys are passed as their raw uint16_t bit patterns. */
+airtopk_status airtopk_select_f32(const float* keys, int64_t batch, int64_t len, int64_t k, int select_min,
+                                  float* out_vals, int64_t* out_idx, airtopk_stream_t stream);
+airtopk_status airtopk_select_f16(const uint16_t* keys, int64_t batch, int64_t len, int64_t k, int select_min,
+                                  uint16_t* out_vals, int64_t* out_idx, airtopk_stream_t stream);
+airtopk_status airtopk_select_bf16(const uint16_t* keys, int64_t batch, int64_t len, int64_t k, int select_min,
+                                   uint16_t* out_vals, int64_t* out_idx, airtopk_stream_t stream);
+airtopk_status airtopk_select_f64(const double* keys, int64_t batch, int64_t len, int64_t k, int select_min,
+                                  double* out_vals, int64_t* out_idx, airtopk_stream_t stream);
+airtopk_status airtopk_select_u32(const uint32_t* keys, int64_t batch, int64_t len, int64_t k, int select_min,
+                                  uint32_t* out_vals, int64_t* out_idx, airtopk_stream_t stream);
+
+/* Merge select for candidates gathered from several GPUs: a single row of
+ * `len` keys whose elements carry caller-given index VALUES in_idx[len] (device, int64, distinct,
+ * each in [0, 2^idx_bits)). Selects the K smallest (largest) keys, ties by smallest in_idx value;
+ * out_idx receives in_idx values. idx_bits in [1, 63]. */
+size_t airtopk_workspace_bytes_with_idx(airtopk_dtype dtype, int64_t len, int64_t k, int idx_bits);
+airtopk_status airtopk_select_with_idx(const void* keys, const int64_t* in_idx, int idx_bits,
+                                       airtopk_dtype dtype, int64_t len, int64_t k, int select_min,
+                                       void* out_vals, int64_t* out_idx, void* workspace,
+                                       size_t workspace_bytes, airtopk_stream_t stream);
+
+/* End-to-end convenience with HOST buffers: copies keys host->device, selects, copies the results
+ * device->host and SYNCHRONISES `stream` before returning. Pinned (page-locked) host memory gives
+ * asynchronous DMA; pageable memory works but is staged by the driver. Device scratch comes from
+ * cudaMallocAsync on `stream`. */
+airtopk_status airtopk_select_host(const void* h_keys, airtopk_dtype dtype, int64_t batch, int64_t len,
+                                   int64_t k, int select_min, void* h_out_vals, int64_t* h_out_idx,
+                                   airtopk_stream_t stream);
+
+/* Human-readable status; never NULL. */
+const char* airtopk_status_str(airtopk_status s);
+/* cudaError_t (as int) of the most recent AIRTOPK_ECUDA on this thread; 0 if none. */
+int airtopk_last_cuda_error(void);
+/* Library version, e.g. "0.1.0". */
+const char* airtopk_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* AIRTOPK_H_ */

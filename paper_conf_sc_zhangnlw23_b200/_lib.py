@@ -1,0 +1,77 @@
+"""ctypes binding of libairtopk.so (include/airtopk.h). Argument marshalling only.
+
+There is deliberately no fallback: if the CUDA library is missing the import fails loudly.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libairtopk.so")
+
+OK, EINVAL, EDTYPE, ENOSPACE, ECUDA = 0, 1, 2, 3, 4
+F32, F16, BF16, F64, U32 = 0, 1, 2, 3, 4
+ENGINE_AUTO, ENGINE_GRID, ENGINE_CLUSTER = 0, 1, 2
+TRACE_MAX_PASSES = 16
+TRACE_FIELDS = ("width", "src_L", "stored", "j", "K", "C", "Cp", "emitted", "early_stop", "read")
+
+# Every symbol include/airtopk.h declares (checked by tests/test_abi.py).
+EXPORTS = (
+    "airtopk_workspace_bytes", "airtopk_workspace_bytes_ex", "airtopk_select", "airtopk_select_ex",
+    "airtopk_select_f32", "airtopk_select_f16", "airtopk_select_bf16", "airtopk_select_f64",
+    "airtopk_select_u32", "airtopk_workspace_bytes_with_idx", "airtopk_select_with_idx",
+    "airtopk_select_host", "airtopk_status_str", "airtopk_last_cuda_error", "airtopk_version",
+)
+
+
+class Options(ctypes.Structure):
+    _fields_ = [
+        ("alpha", ctypes.c_int64),
+        ("engine", ctypes.c_int32),
+        ("ctas_per_row", ctypes.c_int32),
+        ("cluster_size", ctypes.c_int32),
+        ("n_events", ctypes.c_int32),
+        ("trace", ctypes.c_void_p),
+        ("events", ctypes.c_void_p),
+    ]
+
+
+class AirTopKError(RuntimeError):
+    def __init__(self, status: int, lib=None):
+        msg = lib.airtopk_status_str(status).decode() if lib is not None else f"status {status}"
+        if status == ECUDA and lib is not None:
+            msg += f" (cudaError {lib.airtopk_last_cuda_error()})"
+        super().__init__(msg)
+        self.status = status
+
+
+def load(path: str = LIB_PATH):
+    if not os.path.exists(path):
+        raise ImportError(f"{path} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "
+                          "or `python -m paper_conf_sc_zhangnlw23_b200._build` (no CPU fallback exists)")
+    lib = ctypes.CDLL(path)
+    i64, vp, ci, sz = ctypes.c_int64, ctypes.c_void_p, ctypes.c_int, ctypes.c_size_t
+    lib.airtopk_workspace_bytes.argtypes = [ci, i64, i64, i64]
+    lib.airtopk_workspace_bytes.restype = sz
+    lib.airtopk_workspace_bytes_ex.argtypes = [ci, i64, i64, i64, ctypes.POINTER(Options)]
+    lib.airtopk_workspace_bytes_ex.restype = sz
+    lib.airtopk_select.argtypes = [vp, ci, i64, i64, i64, ci, vp, vp, vp, sz, vp]
+    lib.airtopk_select.restype = ci
+    lib.airtopk_select_ex.argtypes = [vp, ci, i64, i64, i64, ci, vp, vp, vp, sz, vp, ctypes.POINTER(Options)]
+    lib.airtopk_select_ex.restype = ci
+    for n in ("airtopk_select_f32", "airtopk_select_f16", "airtopk_select_bf16", "airtopk_select_f64",
+              "airtopk_select_u32"):
+        getattr(lib, n).argtypes = [vp, i64, i64, i64, ci, vp, vp, vp]
+        getattr(lib, n).restype = ci
+    lib.airtopk_workspace_bytes_with_idx.argtypes = [ci, i64, i64, ci]
+    lib.airtopk_workspace_bytes_with_idx.restype = sz
+    lib.airtopk_select_with_idx.argtypes = [vp, vp, ci, ci, i64, i64, ci, vp, vp, vp, sz, vp]
+    lib.airtopk_select_with_idx.restype = ci
+    lib.airtopk_select_host.argtypes = [vp, ci, i64, i64, i64, ci, vp, vp, vp]
+    lib.airtopk_select_host.restype = ci
+    lib.airtopk_status_str.argtypes = [ci]
+    lib.airtopk_status_str.restype = ctypes.c_char_p
+    lib.airtopk_last_cuda_error.restype = ci
+    lib.airtopk_version.restype = ctypes.c_char_p
+    return lib

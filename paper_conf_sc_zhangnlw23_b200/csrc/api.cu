@@ -1,0 +1,279 @@
+// api.cu — the C ABI of libairtopk.so (declared and documented in include/airtopk.h).
+//
+// Argument validation (K in [1, N]), dtype dispatch, workspace carve-up and launch
+// sequencing. Every entry point except airtopk_select_host only enqueues work on the caller's
+// stream (the iteration-fused property: the CPU only launches kernels, P:50/P:142/P:158).
+#include <algorithm>
+#include <cstdlib>
+#include <cstring>
+
+#include "../../include/airtopk.h"
+#include "device.cuh"
+#include "engine.h"
+
+namespace airtopk {
+
+namespace {
+thread_local int g_last_cuda_error = 0;
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+int bits_needed(uint64_t v) {  // number of bits to represent v (0 for v == 0)
+  int b = 0;
+  while (v) { ++b; v >>= 1; }
+  return b;
+}
+
+int num_sms() {
+  static thread_local int dev_cached = -1, sms_cached = 148;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return 148;
+  if (dev != dev_cached) {
+    int n = 0;
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && n > 0) sms_cached = n;
+    dev_cached = dev;
+  }
+  return sms_cached;
+}
+}  // namespace
+
+int key_bits(int kind) {
+  switch (kind) {
+    case K_F32: return 32;
+    case K_F16: return 16;
+    case K_BF16: return 16;
+    case K_F64: return 64;
+    case K_U32: return 32;
+  }
+  return -1;
+}
+
+int key_bytes(int kind) { return key_bits(kind) / 8; }
+
+int grid_vec_chunk(int kind);
+
+// Workspace layout (all offsets 256-aligned):
+//   [RowState x batch][2 histograms x 2048 counters x batch][code buffers 2 x batch x cap][index buffers]
+Plan make_plan(const SelectArgs& a) {
+  Plan p{};
+  p.R = key_bits(a.kind);
+  if (!a.in_idx && a.k == a.len) {
+    p.engine = 3;
+    return p;
+  }
+  p.idx64 = (a.in_idx != nullptr) || (a.len > (int64_t(1) << 32));
+  p.IB = a.in_idx ? a.idx_bits : bits_needed((uint64_t)(a.len - 1));
+  p.P = code_passes(p.R) + idx_passes(p.IB);
+  const int64_t alpha = a.alpha > 0 ? a.alpha : 128;
+  p.cap_rule = (a.len - 1) / alpha;                   // C * alpha < N  <=>  C <= (N-1)/alpha
+  p.cap_alloc = (int64_t)align_up((size_t)p.cap_rule, 8);
+  p.engine = 1;
+  const size_t isz = p.idx64 ? 8 : 4;
+  const size_t csz = isz;  // histogram counter width
+  p.off_state = 0;
+  p.off_hist = align_up(sizeof(RowState) * (size_t)a.batch, 256);
+  p.off_bcode = p.off_hist + align_up((size_t)a.batch * 2 * kMaxBins * csz, 256);
+  p.off_bidx = p.off_bcode + align_up((size_t)2 * a.batch * p.cap_alloc * key_bytes(a.kind), 256);
+  p.bytes = p.off_bidx + align_up((size_t)2 * a.batch * p.cap_alloc * isz, 256);
+  return p;
+}
+
+static void choose_launch(const SelectArgs& a, Plan& p) {
+  if (p.engine != 1) return;
+  if (a.ctas_per_row > 0) {
+    p.cpr = a.ctas_per_row;
+    return;
+  }
+  const int64_t target = (int64_t)num_sms() * grid_blocks_per_sm(a, p.idx64);
+  const int64_t chunk = grid_vec_chunk(a.kind);
+  const int64_t maxc = std::max<int64_t>(1, (a.len + chunk - 1) / chunk);
+  int64_t c = (target + a.batch - 1) / a.batch;
+  p.cpr = (int)std::max<int64_t>(1, std::min<int64_t>(c, maxc));
+}
+
+static bool valid_kind(int dt) { return dt >= AIRTOPK_F32 && dt <= AIRTOPK_U32; }
+
+static airtopk_status validate(const SelectArgs& a) {
+  if (!valid_kind(a.kind)) return AIRTOPK_EDTYPE;
+  if (!a.keys || !a.out_vals || !a.out_idx) return AIRTOPK_EINVAL;
+  if (a.batch < 1 || a.len < 1 || a.k < 1 || a.k > a.len) return AIRTOPK_EINVAL;
+  if (a.alpha < 0) return AIRTOPK_EINVAL;
+  if (a.in_idx && (a.batch != 1 || a.idx_bits < 1 || a.idx_bits > 63)) return AIRTOPK_EINVAL;
+  return AIRTOPK_OK;
+}
+
+static airtopk_status fail_cuda(cudaError_t e) {
+  g_last_cuda_error = (int)e;
+  return AIRTOPK_ECUDA;
+}
+
+static airtopk_status run(const SelectArgs& a, void* ws, size_t ws_bytes, cudaStream_t s) {
+  airtopk_status st = validate(a);
+  if (st != AIRTOPK_OK) return st;
+  Plan p = make_plan(a);
+  if (p.engine == 3) {
+    cudaError_t e = run_trivial(a, s);
+    return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
+  }
+  if (!ws || ws_bytes < p.bytes) return AIRTOPK_ENOSPACE;
+  if (((uintptr_t)ws & 255u) != 0) return AIRTOPK_EINVAL;
+  choose_launch(a, p);
+  cudaError_t e = run_grid(a, p, ws, s);
+  return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
+}
+
+static SelectArgs make_args(const void* keys, int dt, int64_t batch, int64_t len, int64_t k, int select_min,
+                            void* out_vals, int64_t* out_idx, const airtopk_options* opt) {
+  SelectArgs a;
+  a.keys = keys;
+  a.kind = dt;
+  a.batch = batch;
+  a.len = len;
+  a.k = k;
+  a.sel_min = select_min ? 1 : 0;
+  a.out_vals = out_vals;
+  a.out_idx = out_idx;
+  if (opt) {
+    a.alpha = opt->alpha;
+    a.engine = opt->engine;
+    a.ctas_per_row = opt->ctas_per_row;
+    a.cluster_size = opt->cluster_size;
+    a.trace = opt->trace;
+    a.events = opt->events;
+    a.n_events = opt->events ? opt->n_events : 0;
+  }
+  if (a.alpha == 0) a.alpha = 128;
+  return a;
+}
+
+static airtopk_status run_pooled(const SelectArgs& a, cudaStream_t s) {
+  airtopk_status st = validate(a);
+  if (st != AIRTOPK_OK) return st;
+  Plan p = make_plan(a);
+  void* ws = nullptr;
+  if (p.engine != 3 && p.bytes) {
+    cudaError_t e = cudaMallocAsync(&ws, p.bytes, s);
+    if (e != cudaSuccess) return fail_cuda(e);
+  }
+  st = run(a, ws, p.bytes, s);
+  if (ws) {
+    cudaError_t e = cudaFreeAsync(ws, s);
+    if (e != cudaSuccess && st == AIRTOPK_OK) st = fail_cuda(e);
+  }
+  return st;
+}
+
+}  // namespace airtopk
+
+using namespace airtopk;
+
+extern "C" {
+
+size_t airtopk_workspace_bytes_ex(airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k,
+                                  const airtopk_options* opt) {
+  int64_t dummy_out = 0;
+  SelectArgs a = make_args((const void*)1, (int)dtype, batch, len, k, 1, (void*)1, &dummy_out, opt);
+  if (validate(a) != AIRTOPK_OK) return 0;
+  Plan p = make_plan(a);
+  return p.engine == 3 ? 0 : p.bytes;
+}
+
+size_t airtopk_workspace_bytes(airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k) {
+  return airtopk_workspace_bytes_ex(dtype, batch, len, k, nullptr);
+}
+
+airtopk_status airtopk_select_ex(const void* keys, airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k,
+                                 int select_min, void* out_vals, int64_t* out_idx, void* workspace,
+                                 size_t workspace_bytes, airtopk_stream_t stream, const airtopk_options* opt) {
+  SelectArgs a = make_args(keys, (int)dtype, batch, len, k, select_min, out_vals, out_idx, opt);
+  return run(a, workspace, workspace_bytes, (cudaStream_t)stream);
+}
+
+airtopk_status airtopk_select(const void* keys, airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k,
+                              int select_min, void* out_vals, int64_t* out_idx, void* workspace,
+                              size_t workspace_bytes, airtopk_stream_t stream) {
+  return airtopk_select_ex(keys, dtype, batch, len, k, select_min, out_vals, out_idx, workspace, workspace_bytes,
+                           stream, nullptr);
+}
+
+#define AIRTOPK_TYPED(NAME, T, DT)                                                                        \
+  airtopk_status NAME(const T* keys, int64_t batch, int64_t len, int64_t k, int select_min, T* out_vals,  \
+                      int64_t* out_idx, airtopk_stream_t stream) {                                        \
+    SelectArgs a = make_args(keys, DT, batch, len, k, select_min, out_vals, out_idx, nullptr);            \
+    return run_pooled(a, (cudaStream_t)stream);                                                           \
+  }
+
+AIRTOPK_TYPED(airtopk_select_f32, float, AIRTOPK_F32)
+AIRTOPK_TYPED(airtopk_select_f16, uint16_t, AIRTOPK_F16)
+AIRTOPK_TYPED(airtopk_select_bf16, uint16_t, AIRTOPK_BF16)
+AIRTOPK_TYPED(airtopk_select_f64, double, AIRTOPK_F64)
+AIRTOPK_TYPED(airtopk_select_u32, uint32_t, AIRTOPK_U32)
+#undef AIRTOPK_TYPED
+
+size_t airtopk_workspace_bytes_with_idx(airtopk_dtype dtype, int64_t len, int64_t k, int idx_bits) {
+  int64_t dummy = 0;
+  SelectArgs a = make_args((const void*)1, (int)dtype, 1, len, k, 1, (void*)1, &dummy, nullptr);
+  a.in_idx = &dummy;
+  a.idx_bits = idx_bits;
+  if (validate(a) != AIRTOPK_OK) return 0;
+  return make_plan(a).bytes;
+}
+
+airtopk_status airtopk_select_with_idx(const void* keys, const int64_t* in_idx, int idx_bits, airtopk_dtype dtype,
+                                       int64_t len, int64_t k, int select_min, void* out_vals, int64_t* out_idx,
+                                       void* workspace, size_t workspace_bytes, airtopk_stream_t stream) {
+  if (!in_idx) return AIRTOPK_EINVAL;
+  SelectArgs a = make_args(keys, (int)dtype, 1, len, k, select_min, out_vals, out_idx, nullptr);
+  a.in_idx = in_idx;
+  a.idx_bits = idx_bits;
+  return run(a, workspace, workspace_bytes, (cudaStream_t)stream);
+}
+
+airtopk_status airtopk_select_host(const void* h_keys, airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k,
+                                   int select_min, void* h_out_vals, int64_t* h_out_idx, airtopk_stream_t stream) {
+  if (!h_keys || !h_out_vals || !h_out_idx) return AIRTOPK_EINVAL;
+  if (!valid_kind((int)dtype)) return AIRTOPK_EDTYPE;
+  if (batch < 1 || len < 1 || k < 1 || k > len) return AIRTOPK_EINVAL;
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t es = key_bytes((int)dtype);
+  const size_t in_b = (size_t)batch * len * es, ov_b = (size_t)batch * k * es, oi_b = (size_t)batch * k * 8;
+  SelectArgs a = make_args(nullptr, (int)dtype, batch, len, k, select_min, nullptr, nullptr, nullptr);
+  Plan p = make_plan(a);
+  const size_t ws_b = p.engine == 3 ? 0 : p.bytes;
+  const size_t o1 = align_up(in_b, 256), o2 = o1 + align_up(ov_b, 256), o3 = o2 + align_up(oi_b, 256);
+  char* d = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&d, o3 + ws_b, s);
+  if (e != cudaSuccess) return fail_cuda(e);
+  airtopk_status st = AIRTOPK_OK;
+  if ((e = cudaMemcpyAsync(d, h_keys, in_b, cudaMemcpyHostToDevice, s)) != cudaSuccess) st = fail_cuda(e);
+  if (st == AIRTOPK_OK) {
+    a.keys = d;
+    a.out_vals = d + o1;
+    a.out_idx = (int64_t*)(d + o2);
+    st = run(a, ws_b ? d + o3 : nullptr, ws_b, s);
+  }
+  if (st == AIRTOPK_OK && (e = cudaMemcpyAsync(h_out_vals, d + o1, ov_b, cudaMemcpyDeviceToHost, s)) != cudaSuccess)
+    st = fail_cuda(e);
+  if (st == AIRTOPK_OK && (e = cudaMemcpyAsync(h_out_idx, d + o2, oi_b, cudaMemcpyDeviceToHost, s)) != cudaSuccess)
+    st = fail_cuda(e);
+  cudaFreeAsync(d, s);
+  if ((e = cudaStreamSynchronize(s)) != cudaSuccess && st == AIRTOPK_OK) st = fail_cuda(e);
+  return st;
+}
+
+const char* airtopk_status_str(airtopk_status s) {
+  switch (s) {
+    case AIRTOPK_OK: return "AIRTOPK_OK: success";
+    case AIRTOPK_EINVAL: return "AIRTOPK_EINVAL: invalid argument (null pointer, batch/len/k out of range, k > len)";
+    case AIRTOPK_EDTYPE: return "AIRTOPK_EDTYPE: unknown dtype";
+    case AIRTOPK_ENOSPACE: return "AIRTOPK_ENOSPACE: workspace too small";
+    case AIRTOPK_ECUDA: return "AIRTOPK_ECUDA: CUDA error (see airtopk_last_cuda_error)";
+  }
+  return "AIRTOPK: unknown status";
+}
+
+int airtopk_last_cuda_error(void) { return g_last_cuda_error; }
+
+const char* airtopk_version(void) { return "0.1.0"; }
+
+}  // extern "C"

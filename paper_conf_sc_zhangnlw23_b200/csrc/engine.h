@@ -1,0 +1,51 @@
+// engine.h — internal (non-ABI) interface between the C-ABI layer (api.cu) and the engines.
+#pragma once
+
+#include <cstddef>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace airtopk {
+
+struct SelectArgs {
+  const void* keys = nullptr;
+  const int64_t* in_idx = nullptr;  // with_idx variant: caller-given index values (else positions)
+  int idx_bits = 0;                 // with_idx variant: index value width
+  int kind = 0;                     // Kind
+  int64_t batch = 0, len = 0, k = 0;
+  int sel_min = 1;
+  void* out_vals = nullptr;
+  int64_t* out_idx = nullptr;
+  int64_t alpha = 128;
+  int engine = 0;
+  int ctas_per_row = 0;
+  int cluster_size = 0;
+  int64_t* trace = nullptr;
+  void* const* events = nullptr;    // optional cudaEvent_t[n_events] recorded around launches
+  int n_events = 0;
+};
+
+// Resolved launch plan (host side).
+struct Plan {
+  int engine;        // 1 grid, 2 cluster, 3 trivial copy (K == N)
+  int idx64;         // 64-bit internal indices
+  int R;             // key bits
+  int IB;            // index bits appended to the key for the lowest-index tie-break
+  int P;             // radix passes (code + index digits)
+  int64_t cap_rule;  // buffer iff C <= cap_rule  (== C * alpha < N)
+  int64_t cap_alloc; // entries allocated per candidate buffer
+  int cpr;           // CTAs per row (grid engine)
+  int csize;         // CTAs per cluster (cluster engine)
+  size_t off_state, off_hist, off_bcode, off_bidx, bytes;
+};
+
+int key_bits(int kind);
+int key_bytes(int kind);
+Plan make_plan(const SelectArgs& a);
+cudaError_t run_grid(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
+cudaError_t run_cluster(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
+cudaError_t run_trivial(const SelectArgs& a, cudaStream_t s);
+int grid_blocks_per_sm(const SelectArgs& a, int idx64);
+int cluster_engine_ok(const SelectArgs& a, int csize);
+
+}  // namespace airtopk

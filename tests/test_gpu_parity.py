@@ -1,0 +1,237 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, bit-exact.
+
+The bar (BASELINE.json north_star): identical value multiset and identical index set under the
+lowest-index tie rule, on seeded synthetic inputs shaped like the paper's workloads (PAPER.md:231,
+235-241), plus the edge cases the method has (K = 1, K = N, ties straddling K, early stop,
+never/always buffering, misaligned rows, every key type).
+"""
+import numpy as np
+import pytest
+
+import gen
+import oracle
+from helpers import assert_parity, gpu_select, to_device, to_bits
+
+pytestmark = pytest.mark.gpu
+
+
+def _keys(dist, seed, batch, n, m=20):
+    return gen.keys(dist, seed, batch * n, m_bits=m).reshape(batch, n)
+
+
+# ---------------------------------------------------------------- the five BASELINE configs
+
+def test_c1_full():
+    x = gen.config_keys("c1")
+    v, i = gpu_select(x, "f32", 32)
+    assert_parity(x, "f32", 32, True, v, i)
+
+
+def test_c2_full():
+    x = gen.config_keys("c2")
+    v, i = gpu_select(x, "f32", 256)
+    assert_parity(x, "f32", 256, True, v, i)
+
+
+def test_c4_full_adversarial_ties():
+    x = gen.config_keys("c4")
+    v, i = gpu_select(x, "f32", 50000)
+    # closed form: every result is 1.0f and the indices are the first 50,000
+    # positions holding 1.0f
+    first = np.flatnonzero(x[0] == np.float32(1.0))[:50000]
+    assert np.all(v.view(np.uint32) == 0x3F800000)
+    assert np.array_equal(np.sort(i[0]), first)
+    assert_parity(x, "f32", 50000, True, v, i)
+
+
+def test_c3_full():
+    x = gen.config_keys("c3")
+    v, i = gpu_select(x, "f32", 1 << 20)
+    assert_parity(x, "f32", 1 << 20, True, v, i)
+
+
+def test_c5_shard_full():
+    """One 2^30 shard of the c5 row (global indices 2^30 .. 2^31-1) with K = 2^16."""
+    n = 1 << 30
+    x = gen.uniform_f32(gen.config_seed("c5"), n, offset=n)
+    v, i = gpu_select(x, "f32", 1 << 16)
+    assert_parity(x, "f32", 1 << 16, True, v, i)
+
+
+# ---------------------------------------------------------------- distributions x shapes
+
+@pytest.mark.parametrize("dist", ["uniform", "normal", "adversarial"])
+@pytest.mark.parametrize("batch,n,k", [(1, 1 << 20, 1), (1, 1 << 20, 1000), (3, 100003, 4097),
+                                       (100, 1 << 14, 256), (7, 5000, 5000 - 1), (1, 1 << 22, 1 << 12)])
+@pytest.mark.parametrize("select_min", [True, False])
+def test_distributions(dist, batch, n, k, select_min):
+    x = _keys(dist, 123, batch, n)
+    v, i = gpu_select(x, "f32", k, select_min)
+    assert_parity(x, "f32", k, select_min, v, i)
+
+
+@pytest.mark.parametrize("m", [10, 20, 28, 31, 32])
+def test_adversarial_prefix_lengths(m):
+    x = _keys("adversarial", 9, 2, 1 << 18, m)
+    for k in (1, 77, 30000):
+        v, i = gpu_select(x, "f32", k)
+        assert_parity(x, "f32", k, True, v, i)
+
+
+# ---------------------------------------------------------------- edge cases
+
+@pytest.mark.parametrize("n", [1, 2, 3, 31, 32, 33, 255, 1000, 4097, 65537])
+def test_small_and_ragged(n):
+    x = gen.uniform_f32(5, n)
+    for k in sorted({1, max(1, n // 2), max(1, n - 1), n}):
+        v, i = gpu_select(x, "f32", k)
+        assert_parity(x, "f32", k, True, v, i)
+
+
+@pytest.mark.parametrize("off", [1, 2, 3])
+def test_misaligned_rows(off):
+    x = _keys("normal", 4, 3, 7777)
+    v, i = gpu_select(x, "f32", 100, offset_elems=off)
+    assert_parity(x, "f32", 100, True, v, i)
+
+
+def test_all_equal_and_two_valued():
+    x = np.full((2, 100000), 2.5, np.float32)
+    v, i = gpu_select(x, "f32", 1234)
+    assert np.array_equal(np.sort(i, axis=1), np.tile(np.arange(1234), (2, 1)))
+    y = np.where(gen.u32(1, 300000) & 1, np.float32(1), np.float32(2)).astype(np.float32)
+    for k in (1, 1000, 150000, 200000):
+        v, i = gpu_select(y, "f32", k)
+        assert_parity(y, "f32", k, True, v, i)
+
+
+def test_special_values():
+    bits = gen.u32(77, 200000)
+    pool = np.array([0x00000000, 0x80000000, 0x7F800000, 0xFF800000, 0x7FC00000, 0xFFC00001, 0x00000001,
+                     0x80000001, 0x7F7FFFFF, 0xFF7FFFFF, 0x3F800000, 0xBF800000], np.uint32)
+    raw = np.where(bits % 3 == 0, pool[bits % pool.size], bits)
+    for k in (1, 13, 5000, 199999):
+        for sm in (True, False):
+            v, i = gpu_select(raw, "f32", k, sm)
+            assert_parity(raw, "f32", k, sm, v, i)
+
+
+@pytest.mark.parametrize("dtn", ["f16", "bf16", "f64", "u32"])
+@pytest.mark.parametrize("pool", [0, 5])
+def test_other_dtypes(dtn, pool):
+    n = 300001
+    u = gen.u64(31, n)
+    if pool:
+        u = gen.u64(32, pool)[u % np.uint64(pool)]
+    raw = u.astype({"f16": np.uint16, "bf16": np.uint16, "f64": np.uint64, "u32": np.uint32}[dtn])
+    for k in (1, 999, 150000):
+        for sm in (True, False):
+            v, i = gpu_select(raw, dtn, k, sm)
+            assert_parity(raw, dtn, k, sm, v, i)
+
+
+def test_f16_exhaustive():
+    raw = np.arange(1 << 16, dtype=np.uint32).astype(np.uint16)
+    raw = raw[np.argsort(gen.u32(3, 1 << 16))]
+    for k in (1, 1024, 40000, 65535):
+        v, i = gpu_select(raw, "f16", k)
+        assert_parity(raw, "f16", k, True, v, i)
+
+
+# ---------------------------------------------------------------- adaptive strategy / engine knobs
+
+@pytest.mark.parametrize("alpha", [1, 4, 128, 1 << 40])
+@pytest.mark.parametrize("dist,m", [("uniform", 20), ("adversarial", 20), ("adversarial", 10)])
+def test_alpha_invariance(alpha, dist, m):
+    """Results are independent of alpha: always / default / never buffering."""
+    x = _keys(dist, 21, 2, 1 << 20, m)
+    for k in (5, 3000):
+        v, i = gpu_select(x, "f32", k, alpha=alpha)
+        assert_parity(x, "f32", k, True, v, i)
+
+
+@pytest.mark.parametrize("cpr", [1, 2, 7, 300])
+def test_ctas_per_row(cpr):
+    x = _keys("uniform", 8, 3, 200000)
+    v, i = gpu_select(x, "f32", 500, ctas_per_row=cpr)
+    assert_parity(x, "f32", 500, True, v, i)
+
+
+# ---------------------------------------------------------------- per-pass state vs the oracle's Algorithm 1 trace
+
+@pytest.mark.parametrize("dist,m,k,alpha", [("uniform", 20, 1000, 128), ("normal", 20, 77, 128),
+                                            ("adversarial", 20, 5000, 128), ("adversarial", 10, 100, 4),
+                                            ("uniform", 20, 1 << 12, 1 << 40)])
+def test_trace_matches_algorithm1(dist, m, k, alpha):
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    n = 1 << 20
+    x = gen.keys(dist, 55, n, m_bits=m)
+    tr = at.trace_buffer(1)
+    xd = to_device(x, "f32").reshape(1, -1)
+    at.select(xd, k, alpha=alpha, trace=tr, engine=at.ENGINE_GRID)
+    torch.cuda.synchronize()
+    g = tr.cpu().numpy()[0]
+    codes = oracle.codes(x)
+    _, recs, _ = oracle.radix_trace(codes, k, r_bits=32, b=11, idx_bits=20, alpha=alpha)
+    emitted = 0
+    for q, r in enumerate(recs[:-1]):
+        t = dict(zip(at._lib.TRACE_FIELDS, g[q].tolist()))
+        emitted += r["emitted"]
+        for f in ("width", "src_L", "stored", "j", "K", "C", "Cp", "early_stop", "read"):
+            assert t[f] == r[f], f"pass {q} field {f}: gpu {t[f]} oracle {r[f]}"
+        assert t["emitted"] == emitted
+    assert g[len(recs) - 1][0] == -1      # no scan after the early stop
+
+
+# ---------------------------------------------------------------- other entry points
+
+def test_with_idx_merge():
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    n, k = 200000, 5000
+    x = gen.adversarial_f32(3, n, m_bits=24)
+    perm = np.argsort(gen.u32(4, n)).astype(np.int64)
+    gid = perm * 3 + 1000                       # distinct, not position-ordered
+    v, i = at.select_with_idx(to_device(x, "f32"), torch.from_numpy(gid).cuda(), k, idx_bits=21)
+    rv, ri = oracle.topk_with_idx(x, gid, k)
+    gi = i.cpu().numpy()
+    assert np.array_equal(np.sort(gi), np.sort(ri))
+    inv = np.full(gid.max() + 1, -1, np.int64)
+    inv[gid] = np.arange(n)
+    assert np.array_equal(to_bits(v, "f32"), x[inv[gi]].view(np.uint32))
+
+
+def test_select_host_e2e():
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    x = gen.config_keys("c2", batch=10)
+    xt = torch.from_numpy(x).pin_memory()
+    v, i = at.select_host(xt, 256)
+    assert_parity(x, "f32", 256, True, v.numpy().view(np.uint32), i.numpy())
+
+
+def test_typed_entry_points_pool_workspace():
+    import ctypes
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    x = gen.config_keys("c1")
+    xd = to_device(x, "f32")
+    v = torch.empty((1, 32), dtype=torch.float32, device="cuda")
+    i = torch.empty((1, 32), dtype=torch.int64, device="cuda")
+    s = torch.cuda.current_stream().cuda_stream
+    assert at.lib().airtopk_select_f32(xd.data_ptr(), 1, x.shape[1], 32, 1, v.data_ptr(), i.data_ptr(), s) == 0
+    torch.cuda.synchronize()
+    assert_parity(x, "f32", 32, True, to_bits(v, "f32"), i.cpu().numpy())
+
+
+def test_repeated_calls_reuse_workspace():
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    x = _keys("normal", 70, 4, 1 << 16)
+    xd = to_device(x, "f32")
+    ws = torch.empty(at.workspace_bytes(torch.float32, 4, 1 << 16, 300), dtype=torch.uint8, device="cuda")
+    for _ in range(3):
+        v, i = at.select(xd, 300, workspace=ws)
+    torch.cuda.synchronize()
+    assert_parity(x, "f32", 300, True, to_bits(v, "f32"), i.cpu().numpy())
