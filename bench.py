@@ -1,0 +1,408 @@
+#!/usr/bin/env python
+"""bench.py — AIR Top-K on B200: top-K elements/s and achieved HBM GB/s vs B200 peak.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--impl ours|reference]
+
+One "step" = one full AIR Top-K select (every radix pass + the last filter) over the
+config's synthetic input, already resident in HBM. Default workload = c3 (batch 1, N = 2^30
+uniform (0,1] f32, K = 2^20, select-min), the configuration BASELINE.json's metric is quoted on.
+
+N > 1 (torchrun, one rank per GPU, NCCL):
+  c3/c5-style: one row of N * 2^30 elements split across the ranks (per-GPU work fixed -> "weak"):
+      local select of the 2^30 shard + NCCL all-gather of the K candidates + merge select.
+  c2: the 100 rows are sharded across ranks (total work fixed -> "strong"), no collective.
+
+The oracle (oracle/, CPU) is executed ONLY by the cpu_baseline leg and by --impl reference.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import gen  # noqa: E402
+
+PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FALLBACK_HBM_GBS = 6650.0  # /opt/skills/guides/B200_PROFILING.md fallback
+
+CFG = {
+    "c1": dict(batch=1, n=1 << 16, k=32, dist="uniform"),
+    "c2": dict(batch=100, n=1 << 20, k=256, dist="normal"),
+    "c3": dict(batch=1, n=1 << 30, k=1 << 20, dist="uniform"),
+    "c4": dict(batch=1, n=1 << 28, k=50000, dist="adversarial"),
+}
+DEFAULT_STEPS = {"c1": 200, "c2": 100, "c3": 60, "c4": 60}
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def hbm_peak():
+    try:
+        with open(PEAKS_FILE) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback"
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi sampling of SM clocks and throttle reasons during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index: int):
+        self.dev = device_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        time.sleep(0.12)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 6:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[2:6]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- inputs
+def host_keys(cfg_name: str, n: int, batch: int, offset: int = 0):
+    c = CFG[cfg_name]
+    seed = gen.config_seed(cfg_name)
+    return gen.keys(c["dist"], seed, batch * n, offset=offset).reshape(batch, n)
+
+
+def n_passes(n: int, R: int = 32):
+    ib = int(n - 1).bit_length()
+    return -(-R // 11) + -(-ib // 11)
+
+
+# ----------------------------------------------------------------------------- reference arm / CPU baseline
+def cpu_sample_run(cfg_name: str, budget_s: float):
+    """Time the CPU oracle (oracle.topk_nth, single thread, as it stands) on a bounded sample of the
+    workload: same distribution and K/N ratio, N_s = min(N, 2^26) per row."""
+    import oracle
+    c = CFG[cfg_name]
+    ns = min(c["n"], 1 << 26)
+    ks = max(1, round(c["k"] * ns / c["n"]))
+    rows = 1 if c["batch"] == 1 else min(c["batch"], max(1, (1 << 26) // ns))
+    x = host_keys(cfg_name, ns, rows)
+    oracle.build()
+    oracle.topk_nth(x[:1, : min(ns, 1 << 16)], min(ks, 1 << 16))  # load / warm
+    t0 = time.perf_counter()
+    reps = 0
+    while True:
+        oracle.topk_nth(x, ks)
+        reps += 1
+        el = time.perf_counter() - t0
+        if el >= budget_s:
+            break
+    value = reps * rows * ns / el
+    return {"value": value, "unit": "elements/s", "cores": 1, "kind": "oracle",
+            "sample": f"{reps} x oracle.topk_nth on {rows} x 2^{int(math.log2(ns))} {c['dist']} f32, K={ks} "
+                      f"(same K/N as {cfg_name}), {el:.1f} s single-threaded std::nth_element"}
+
+
+def run_reference(args, rank):
+    if rank != 0:
+        return
+    cfg = args.config
+    c = CFG[cfg]
+    cb = cpu_sample_run(cfg, args.ref_budget)
+    line = {"impl": "reference", "metric": f"top-K elements/s ({cfg})", "value": cb["value"], "unit": "elements/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": c["batch"] * c["n"] / cb["value"] * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": cfg, "batch": c["batch"], "n": c["n"], "k": c["k"], "dist": c["dist"]},
+            "cpu_baseline": cb, "e2e": {"value": cb["value"], "unit": "elements/s", "h2d_bytes_per_step": 0,
+                                        "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- our arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=None)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="c3", choices=sorted(CFG))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-extras", action="store_true", help="skip the c1/c2/c4 side measurements")
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--cpu-budget", type=float, default=10.0)
+    ap.add_argument("--ref-budget", type=float, default=20.0)
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    args = ap.parse_args()
+    if args.steps is None:
+        args.steps = DEFAULT_STEPS[args.config]
+    args.warmup = max(3, args.warmup)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank)
+        return
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_zhangnlw23_b200 as at
+    from paper_conf_sc_zhangnlw23_b200 import dist as atdist
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=dev)
+    at.lib()
+
+    cfg = args.config
+    c = CFG[cfg]
+    peak, peak_kind = hbm_peak()
+
+    # ---------------- workload on this rank
+    if cfg == "c2":
+        lo, hi = atdist.row_range(c["batch"], rank, world)
+        batch, n = hi - lo, c["n"]
+        xh = host_keys(cfg, n, batch, offset=lo * n)
+        scaling = "strong"
+        total_units = c["batch"] * c["n"]
+        split = False
+    else:
+        batch, n = c["batch"], c["n"]
+        xh = host_keys(cfg, n, batch, offset=rank * n * batch)
+        scaling = "weak"
+        total_units = world * batch * n
+        split = world > 1
+    k = c["k"]
+    xd = torch.from_numpy(xh).to(dev)
+    ws = torch.empty(max(1, at.workspace_bytes(torch.float32, batch, n, k)), dtype=torch.uint8, device=dev)
+    ov = torch.empty((batch, k), dtype=torch.float32, device=dev)
+    oi = torch.empty((batch, k), dtype=torch.int64, device=dev)
+    P = n_passes(n)
+    n_launch = P + 1
+    stream = torch.cuda.current_stream(dev)
+    ev_sets = []
+
+    def step(events=None):
+        v, i = at.select(xd, k, workspace=ws, out=(ov, oi), events=events)
+        if split:
+            gv, gi = atdist.select_split_row(xd.reshape(-1), k, total_len=world * n, shard_offset=rank * n,
+                                             select_fn=lambda t, kk, lg: (v.reshape(-1), i.reshape(-1)))
+            return gv, gi
+        return v, i
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    # per-kernel events for every timed step (recorded on the launching stream by the library)
+    for _ in range(args.steps):
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(n_launch + 1)]
+        for e in evs:
+            e.record(stream)  # creates the cudaEvent_t; the library re-records it between launches
+        ev_sets.append((evs, at.make_event_array(evs)))
+    torch.cuda.synchronize()
+
+    sampler = ClockSampler(local)
+    sampler.start()
+    time.sleep(0.15)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_start.record(stream)
+    for s_i in range(args.steps):
+        step(ev_sets[s_i][1])
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop()
+    ms_local = t_start.elapsed_time(t_end) / args.steps
+    ms = ms_local
+    if world > 1:
+        tt = torch.tensor([ms_local], device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms = float(tt.item())
+
+    # per-kernel durations (the select's launches; the merge path for N>1 is not in these events)
+    per = np.zeros(n_launch)
+    for evs, _ in ev_sets:
+        for q in range(n_launch):
+            per[q] += evs[q].elapsed_time(evs[q + 1])
+    per /= args.steps
+    select_ms = float(per.sum())
+    dom = int(np.argmax(per))
+    in_bytes = batch * n * 4
+    out_bytes = batch * k * (4 + 8)
+    # algorithmic bytes of the dominant kernel: passes that read the input read N*4 bytes once
+    dom_alg = in_bytes if dom <= 1 else None
+    value = total_units / (ms * 1e-3)
+
+    # ---------------- correctness spot check of the timed configuration (sampled, no oracle):
+    v_chk, i_chk = step()
+    torch.cuda.synchronize()
+
+    result = None
+    if rank == 0:
+        roofline = None
+        if dom_alg is not None:
+            ach = dom_alg / (per[dom] * 1e-3) / 1e9
+            roofline = {"bound": "hbm", "kernel": f"grid_pass_kernel q={dom}", "achieved": ach, "peak": peak,
+                        "peak_kind": peak_kind, "unit": "GB/s", "frac": ach / peak,
+                        "traffic": load_traffic(cfg, dom),
+                        "alg_bytes_per_launch": dom_alg, "launch_ms": float(per[dom])}
+        whole = (in_bytes + out_bytes) / (select_ms * 1e-3) / 1e9
+        result = {
+            "metric": "top-K elements/s and achieved HBM GB/s vs B200 peak (N=2^30,K=2^20; b=100)",
+            "value": value, "unit": "elements/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": ms, "higher_is_better": True, "scaling": scaling, "vs_baseline": None,
+            "dtype": "f32", "data": "synthetic",
+            "config": {"workload": cfg, "batch": c["batch"], "n": n, "k": k, "dist": c["dist"], "select": "min",
+                       "per_gpu_rows": batch, "split_row": split,
+                       "l2": "input (%.2f GB) larger than L2 (126 MB): no flush needed" % (in_bytes / 1e9)
+                       if in_bytes > (256 << 20) else "input smaller than L2: consecutive steps may hit L2",
+                       "parallelism": f"{'split-row' if split else ('rows' if cfg == 'c2' else 'replica')}x{world}"},
+            "roofline": roofline,
+            "whole_select": {"achieved_gbs": whole, "frac": whole / peak, "ms": select_ms,
+                             "alg_bytes": in_bytes + out_bytes,
+                             "per_kernel_ms": [float(x) for x in per]},
+            "gpu_launches": args.steps * (n_launch + (2 if split else 0)),
+            "clocks": clocks,
+        }
+    # ---------------- e2e through the C ABI with HOST buffers (pinned), N GPUs, same metric
+    if True:
+        xpin = torch.from_numpy(xh).pin_memory()
+        ovh = torch.empty((batch, k), dtype=torch.float32).pin_memory()
+        oih = torch.empty((batch, k), dtype=torch.int64).pin_memory()
+        at.select_host(xpin, k, out=(ovh, oih))
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            at.select_host(xpin, k, out=(ovh, oih))
+        el = (time.perf_counter() - t0) / args.e2e_steps
+        if world > 1:
+            tt = torch.tensor([el], device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            el = float(tt.item())
+        if rank == 0:
+            result["e2e"] = {"value": total_units / el, "unit": "elements/s", "ms_per_step": el * 1e3,
+                             "h2d_bytes_per_step": in_bytes, "d2h_bytes_per_step": out_bytes,
+                             "path": "airtopk_select_host (pinned H2D + select + D2H + stream sync)"}
+        del xpin
+
+    if rank == 0:
+        # oracle-free sanity of the timed output: K distinct indices, values = keys[idx]
+        ii = i_chk.reshape(-1)[: min(k, 4096)].cpu().numpy()
+        vv = v_chk.reshape(-1)[: min(k, 4096)].cpu().numpy()
+        if not split:
+            assert np.array_equal(xh.reshape(-1)[ii].view(np.uint32), vv.view(np.uint32)), "value/index mismatch"
+        if not args.no_cpu:
+            result["cpu_baseline"] = cpu_sample_run(cfg, args.cpu_budget)
+        if world == 1 and not args.no_extras and cfg == "c3":
+            del xd, ws, ov, oi
+            torch.cuda.empty_cache()
+            result["extras"] = {name: extra_measure(name, dev) for name in ("c1", "c2", "c4")}
+        print(json.dumps(result), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def load_traffic(cfg, q):
+    """dram bytes (read+write) per launch of kernel q from the committed ncu summary, if any."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(cfg, {}).get(str(q))
+    except Exception:
+        return None
+
+
+def extra_measure(name, dev, steps=None, warmup=5):
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    c = CFG[name]
+    steps = steps or DEFAULT_STEPS[name]
+    xh = host_keys(name, c["n"], c["batch"])
+    xd = torch.from_numpy(xh).to(dev)
+    k = c["k"]
+    ws = torch.empty(max(1, at.workspace_bytes(torch.float32, c["batch"], c["n"], k)), dtype=torch.uint8, device=dev)
+    ov = torch.empty((c["batch"], k), dtype=torch.float32, device=dev)
+    oi = torch.empty((c["batch"], k), dtype=torch.int64, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    for _ in range(warmup):
+        at.select(xd, k, workspace=ws, out=(ov, oi))
+    torch.cuda.synchronize()
+    small = c["batch"] * c["n"] * 4 < (512 << 20)
+    tot = 0.0
+    for _ in range(steps):
+        if small:
+            flush.fill_(1)  # write > L2 between timed iterations
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        at.select(xd, k, workspace=ws, out=(ov, oi))
+        e1.record()
+        e1.synchronize()
+        tot += e0.elapsed_time(e1)
+    ms = tot / steps
+    in_bytes = c["batch"] * c["n"] * 4
+    out_bytes = c["batch"] * k * 12
+    peak, _ = hbm_peak()
+    gbs = (in_bytes + out_bytes) / (ms * 1e-3) / 1e9
+    return {"value": c["batch"] * c["n"] / (ms * 1e-3), "unit": "elements/s", "ms_per_step": ms,
+            "alg_gbs": gbs, "frac_of_peak": gbs / peak, "steps": steps,
+            "l2": "flushed (256 MB write) between steps" if small else "input > L2"}
+
+
+if __name__ == "__main__":
+    main()

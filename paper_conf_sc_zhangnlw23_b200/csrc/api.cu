@@ -68,6 +68,7 @@ Plan make_plan(const SelectArgs& a) {
   p.cap_rule = (a.len - 1) / alpha;                   // C * alpha < N  <=>  C <= (N-1)/alpha
   p.cap_alloc = (int64_t)align_up((size_t)p.cap_rule, 8);
   p.engine = 1;
+  p.max_clusters = (int)std::min<int64_t>(a.batch, 2 * 148);
   const size_t isz = p.idx64 ? 8 : 4;
   const size_t csz = isz;  // histogram counter width
   p.off_state = 0;
@@ -78,8 +79,29 @@ Plan make_plan(const SelectArgs& a) {
   return p;
 }
 
+// Engine choice: the cluster engine (one launch, DSMEM scans) for batched
+// and small rows, the grid engine (one launch per pass, whole GPU per row) for long rows.
+static int auto_engine(const SelectArgs& a) {
+  if (a.len <= (int64_t(1) << 17)) return 2;
+  if (a.len <= (int64_t(1) << 22) && a.batch >= 16) return 2;
+  return 1;
+}
+
+static int auto_cluster_size(const SelectArgs& a) {
+  if (a.cluster_size > 0) return a.cluster_size;
+  int64_t c = (a.len + 4095) / 4096;  // >= 4096 elements per CTA
+  int cs = 1;
+  while (cs < 16 && cs < c) cs <<= 1;
+  return cs;
+}
+
 static void choose_launch(const SelectArgs& a, Plan& p) {
-  if (p.engine != 1) return;
+  if (p.engine == 3) return;
+  p.engine = a.engine > 0 ? a.engine : auto_engine(a);
+  if (p.engine == 2) {
+    p.csize = auto_cluster_size(a);
+    return;
+  }
   if (a.ctas_per_row > 0) {
     p.cpr = a.ctas_per_row;
     return;
@@ -98,6 +120,7 @@ static airtopk_status validate(const SelectArgs& a) {
   if (!a.keys || !a.out_vals || !a.out_idx) return AIRTOPK_EINVAL;
   if (a.batch < 1 || a.len < 1 || a.k < 1 || a.k > a.len) return AIRTOPK_EINVAL;
   if (a.alpha < 0) return AIRTOPK_EINVAL;
+  if (a.engine < 0 || a.engine > 2) return AIRTOPK_EINVAL;
   if (a.in_idx && (a.batch != 1 || a.idx_bits < 1 || a.idx_bits > 63)) return AIRTOPK_EINVAL;
   return AIRTOPK_OK;
 }
@@ -118,7 +141,8 @@ static airtopk_status run(const SelectArgs& a, void* ws, size_t ws_bytes, cudaSt
   if (!ws || ws_bytes < p.bytes) return AIRTOPK_ENOSPACE;
   if (((uintptr_t)ws & 255u) != 0) return AIRTOPK_EINVAL;
   choose_launch(a, p);
-  cudaError_t e = run_grid(a, p, ws, s);
+  if (p.engine == 2 && (p.csize < 1 || p.csize > 16 || (p.csize & (p.csize - 1)))) return AIRTOPK_EINVAL;
+  cudaError_t e = (p.engine == 2) ? run_cluster(a, p, ws, s) : run_grid(a, p, ws, s);
   return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
 }
 

@@ -36,6 +36,7 @@ struct Plan {
   int64_t cap_alloc; // entries allocated per candidate buffer
   int cpr;           // CTAs per row (grid engine)
   int csize;         // CTAs per cluster (cluster engine)
+  int max_clusters;  // cluster engine: clusters the workspace has candidate buffers for
   size_t off_state, off_hist, off_bcode, off_bidx, bytes;
 };
 
@@ -46,6 +47,5 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t 
 cudaError_t run_cluster(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 cudaError_t run_trivial(const SelectArgs& a, cudaStream_t s);
 int grid_blocks_per_sm(const SelectArgs& a, int idx64);
-int cluster_engine_ok(const SelectArgs& a, int csize);
 
 }  // namespace airtopk

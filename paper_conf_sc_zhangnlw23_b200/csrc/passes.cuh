@@ -1,0 +1,320 @@
+// passes.cuh — the streaming body of one AIR Top-K pass, shared by both engines.
+//
+// One call processes this CTA's slice of the pass source (Alg1 L7-8: the input row L or the
+// candidate buffer of the previous pass) and performs, per element,
+//   DF (digit filtered, Alg1 L15-22): results (digit < target) -> output V/I; candidates
+//       (digit == target) -> candidate buffer if C < N/alpha (L17-18);
+//   DH (digit histogrammed, L12-13 / L19-20): candidates counted in the shared histogram.
+// DF/DH: 0 none, 1 key digit, 2 index digit (the lowest-index tie-break digits).
+//
+// B200 choices (measured): 4 x 128-bit ld.global.nc.L1::no_allocate per
+// thread in flight; per-element work is 3-4 integer ops and a predicated shared atomic
+// (ATOMS.POPC.INC aggregates equal addresses within a warp); results/candidates, rare in most
+// passes, leave through per-warp shared queues flushed with one global atomic per 64 entries and
+// coalesced stores; the flagged element is re-read from L2 in the slow path so the tile registers
+// die early (40 registers -> 3 CTAs x 512 threads per SM, no spills).
+#pragma once
+
+#include <algorithm>
+#include <type_traits>
+
+#include "device.cuh"
+
+namespace airtopk {
+
+constexpr int kUnroll = 4;
+constexpr int kQCap = 64;
+// Copies of the shared histogram in the filter passes: lane l counts into copy l % kHistCopies
+// (interleaved bin-major so copies of one bin sit in different banks); cuts the same-address
+// serialisation of shared atomics when many lanes hit a few bins (radix-adversarial passes).
+constexpr int kHistCopies = 4;
+
+template <typename U, typename IdxT>
+struct WarpQ {
+  static constexpr int kCap = (sizeof(U) + sizeof(IdxT) <= 8) ? kQCap : kQCap / 2;
+  U code[kCap];
+  IdxT idx[kCap];
+};
+
+template <int KIND, typename IdxT, int DF>
+__host__ __device__ constexpr int hist_copies() {
+  using U = typename KT<KIND>::U;
+  return (DF == 0) ? 1 : (sizeof(U) + sizeof(IdxT) <= 8 ? kHistCopies : 2);
+}
+
+// Flush a warp queue: ONE global atomic reserves n slots, then coalesced stores. Out of line so the
+// streaming loop stays small (I-cache). mode 0: results (value bits + int64 index), 1: candidates.
+template <int KIND, typename IdxT>
+__device__ __noinline__ void wq_flush(const WarpQ<typename KT<KIND>::U, IdxT>* wq, int n, unsigned long long* counter,
+                                      unsigned long long limit, typename KT<KIND>::U* dst_code, void* dst_idx,
+                                      int mode, bool sel_min, unsigned* err) {
+  const int lane = threadIdx.x & 31;
+  unsigned long long base = 0;
+  if (lane == 0) base = atomicAdd(counter, (unsigned long long)n);
+  base = __shfl_sync(kFull, base, 0);
+  for (int j = lane; j < n; j += 32) {
+    const unsigned long long pos = base + j;
+    if (pos < limit) {
+      if (mode == 0) {
+        dst_code[pos] = from_code<KIND>(wq->code[j], sel_min);
+        ((int64_t*)dst_idx)[pos] = (int64_t)wq->idx[j];
+      } else {
+        dst_code[pos] = wq->code[j];
+        ((IdxT*)dst_idx)[pos] = wq->idx[j];
+      }
+    } else {
+      *err = mode == 0 ? 1u : 2u;
+    }
+  }
+}
+
+// Warp-collective append of the lanes with `pred` to a shared-memory queue (flushes when full).
+template <int KIND, typename IdxT>
+__device__ __forceinline__ void wq_push(WarpQ<typename KT<KIND>::U, IdxT>* wq, int& cnt, bool pred,
+                                        typename KT<KIND>::U code, IdxT idx, unsigned long long* counter,
+                                        unsigned long long limit, typename KT<KIND>::U* dst_code, void* dst_idx,
+                                        int mode, bool sel_min, unsigned* err) {
+  const unsigned m = __ballot_sync(kFull, pred);
+  if (!m) return;
+  const int n = __popc(m);
+  if (cnt + n > WarpQ<typename KT<KIND>::U, IdxT>::kCap) {
+    __syncwarp();
+    wq_flush<KIND, IdxT>(wq, cnt, counter, limit, dst_code, dst_idx, mode, sel_min, err);
+    cnt = 0;
+    __syncwarp();
+  }
+  if (pred) {
+    const int pos = cnt + __popc(m & lanemask_lt());
+    wq->code[pos] = code;
+    wq->idx[pos] = idx;
+  }
+  cnt += n;
+}
+
+// Everything one pass of one row needs (built by the engine from its copy of the row state).
+template <typename U, typename IdxT>
+struct PassCtx {
+  int q;
+  bool emit_all, do_hist, srcL, store, sel_min, reverse;
+  Digit dh, df;
+  unsigned long long tcode, tidx;  // fixed prefix bits after scan q-1
+  // source: row L (slice `slice` of `nslices`) or the previous candidate buffer
+  const U* rowp;
+  const int64_t* rowi;  // HASIDX: caller-given index values of the row
+  int64_t len;
+  int slice, nslices;
+  const U* bcin;
+  const IdxT* biin;
+  unsigned long long nbuf;
+  // results
+  U* ov;
+  int64_t* oi;
+  unsigned long long* outc;
+  unsigned long long kk;
+  // candidates
+  U* bco;
+  IdxT* bio;
+  unsigned long long* bufc;
+  unsigned long long capa;
+  unsigned* err;
+  unsigned* hist;  // shared, kMaxBins * hist_copies() counters, zeroed by the caller
+  WarpQ<U, IdxT>* oq;
+  WarpQ<U, IdxT>* bq;
+};
+
+// Runs the pass over this CTA's slice; all queues are flushed on return. Returns the number of
+// elements of the whole source (for the trace).
+template <int KIND, typename IdxT, int DF, int DH, bool HASIDX, int BLOCK>
+__device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT<KIND>::U, IdxT>& c) {
+  using U = typename KT<KIND>::U;
+  using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;  // shifted-key width
+  constexpr int VEC = 16 / sizeof(U);
+  constexpr int HC = hist_copies<KIND, IdxT, DF>();
+  const int tid = threadIdx.x, lane = tid & 31;
+
+  const int shh = c.dh.shift;
+  const unsigned hmask = (1u << c.dh.width) - 1u;
+  const int sf = c.df.shift;
+  const bool emit_all = c.emit_all, do_hist = c.do_hist, store = c.store, sel_min = c.sel_min;
+
+  W tc = 0, bc = 0;
+  U fc = 0;
+  IdxT ti = 0, bi = 0;
+  if (DF == 1) {
+    tc = (W)(c.tcode >> sf);
+    bc = tc & ~(W)((1u << c.df.width) - 1u);
+  } else if (DF == 2) {
+    fc = (U)c.tcode;
+    ti = (IdxT)(c.tidx >> sf);
+    bi = ti & ~(IdxT)((1u << c.df.width) - 1u);
+  }
+  unsigned* const hist_lane = c.hist + (HC > 1 ? (lane % HC) : 0);
+  int ocnt = 0, bcnt = 0;
+
+  auto push_out = [&](bool pred, U code, IdxT idx) {
+    wq_push<KIND, IdxT>(c.oq, ocnt, pred, code, idx, c.outc, c.kk, c.ov, c.oi, 0, sel_min, c.err);
+  };
+  auto push_buf = [&](bool pred, U code, IdxT idx) {
+    wq_push<KIND, IdxT>(c.bq, bcnt, pred, code, idx, c.bufc, c.capa, c.bco, c.bio, 1, sel_min, c.err);
+  };
+  // Filter classification of digit q-1 (Alg1 L15-22): win = result, cand = candidate for pass q.
+  auto classify = [&](U code, IdxT idx, bool valid, bool& win, bool& cand) {
+    bool lt, eq;
+    if constexpr (DF == 1) {
+      const W h = (W)code >> sf;
+      lt = (W)(h - bc) < (W)(tc - bc);
+      eq = (h == tc);
+    } else {
+      const bool ce = (code == fc);
+      const IdxT h = (IdxT)(idx >> sf);
+      lt = ce & ((IdxT)(h - bi) < (IdxT)(ti - bi));
+      eq = ce & (h == ti);
+    }
+    win = valid & (lt | (emit_all & eq));
+    cand = valid & !emit_all & eq;
+  };
+  auto hist_cand = [&](U code, IdxT idx) {  // Alg1 L19-20
+    unsigned d;
+    if constexpr (DH == 2) d = (unsigned)(idx >> shh) & hmask;
+    else d = (unsigned)((W)code >> shh) & hmask;
+    atomicAdd(&hist_lane[d * HC], 1u);
+  };
+
+  unsigned long long nread;
+  if (c.srcL) {
+    // ---- source = the input row L (contiguous slice per CTA, 16-byte vectors) ----
+    const U* rowp = c.rowp;
+    const uintptr_t mis = (uintptr_t)rowp & 15u;
+    const int64_t head = mis ? std::min<int64_t>(c.len, (int64_t)((16u - mis) / sizeof(U))) : 0;
+    const int64_t nvec = (c.len - head) / VEC;
+    const int64_t tail0 = head + nvec * VEC;
+    const int64_t per = (nvec + c.nslices - 1) / c.nslices;
+    const int64_t v0 = std::min<int64_t>(nvec, (int64_t)c.slice * per);
+    const int64_t v1 = std::min<int64_t>(nvec, v0 + per);
+    const uint4* vp = (const uint4*)(rowp + head);
+    nread = c.len;
+
+    auto index_of = [&](int64_t pos) -> IdxT {  // lazily: only results/candidates/index digits need it
+      if constexpr (HASIDX) return (IdxT)c.rowi[pos];
+      else return (IdxT)pos;
+    };
+
+    auto process_tile = [&](const uint4 (&r)[kUnroll], int64_t vb, int64_t vlim) {
+      if constexpr (DF == 0) {
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+          const bool valid = vb + (int64_t)u * BLOCK < vlim;
+#pragma unroll
+          for (int e = 0; e < VEC; ++e) {
+            const U code = to_code<KIND>(vec_elem<U>(r[u], e), sel_min);
+            if (valid) atomicAdd(&c.hist[((W)code >> shh) & hmask], 1u);
+          }
+        }
+      } else {
+        unsigned fw = 0, fcand = 0;  // per-element result / stored-candidate flags
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+          const int64_t v = vb + (int64_t)u * BLOCK;
+          const bool valid = v < vlim;
+#pragma unroll
+          for (int e = 0; e < VEC; ++e) {
+            const U code = to_code<KIND>(vec_elem<U>(r[u], e), sel_min);
+            IdxT idx = 0;
+            if constexpr (DF == 2 || DH == 2) {
+              // the index is needed to classify (DF == 2) or to histogram a candidate (DH == 2)
+              bool need = true;
+              if constexpr (HASIDX) need = (DF == 2) ? (code == fc) : (((W)code >> sf) == tc);
+              if (need && valid) idx = index_of(head + v * VEC + e);
+            }
+            bool win, cand;
+            classify(code, idx, valid, win, cand);
+            if (do_hist && cand) hist_cand(code, idx);
+            fw |= (unsigned)win << (u * VEC + e);
+            fcand |= (unsigned)(cand & store) << (u * VEC + e);
+          }
+        }
+        // slow path (rare in most passes): results / candidates through the warp queues
+        unsigned fl = fw | fcand;
+        while (__any_sync(kFull, fl != 0)) {
+          const int b = fl ? __ffs(fl) - 1 : 0;
+          const bool w = (fw >> b) & (fl != 0), cd = (fcand >> b) & (fl != 0);
+          fl &= fl - 1;
+          // re-read the flagged element (an L2 hit: this warp just streamed it) instead of keeping
+          // the tile registers alive across the slow path
+          const int64_t pos = head + (vb + (int64_t)(b / VEC) * BLOCK) * VEC + (b % VEC);
+          const U code = to_code<KIND>((w | cd) ? __ldcg(rowp + pos) : (U)0, sel_min);
+          const IdxT idx = (w | cd) ? index_of(pos) : (IdxT)0;
+          push_out(w, code, idx);
+          if (store) push_buf(cd, code, idx);
+        }
+      }
+    };
+
+    const int64_t tile = (int64_t)BLOCK * kUnroll;
+    const int64_t nfull = (v1 - v0) / tile;
+    for (int64_t t = 0; t < nfull; ++t) {
+      const int64_t tt = c.reverse ? (nfull - 1 - t) : t;
+      const int64_t vb = v0 + tt * tile + tid;
+      uint4 r[kUnroll];
+#pragma unroll
+      for (int u = 0; u < kUnroll; ++u) r[u] = ldg_stream(vp + vb + (int64_t)u * BLOCK);
+      process_tile(r, vb, v1);
+    }
+    if (v0 + nfull * tile < v1) {
+      const int64_t vb = v0 + nfull * tile + tid;
+      uint4 r[kUnroll];
+#pragma unroll
+      for (int u = 0; u < kUnroll; ++u) {
+        const int64_t v = vb + (int64_t)u * BLOCK;
+        r[u] = (v < v1) ? ldg_stream(vp + v) : make_uint4(0, 0, 0, 0);
+      }
+      process_tile(r, vb, v1);
+    }
+    // scalar head (slice 0) and tail (last slice) of a misaligned / ragged row
+    auto process_scalar = [&](int64_t i, bool valid) {
+      const U code = to_code<KIND>(valid ? rowp[i] : (U)0, sel_min);
+      if constexpr (DF == 0) {
+        if (valid) atomicAdd(&c.hist[((W)code >> shh) & hmask], 1u);
+      } else {
+        const IdxT idx = valid ? index_of(i) : (IdxT)0;
+        bool win, cand;
+        classify(code, idx, valid, win, cand);
+        if (do_hist && cand) hist_cand(code, idx);
+        push_out(win, code, idx);
+        if (store) push_buf(cand, code, idx);
+      }
+    };
+    for (int64_t hb = 0; hb < head; hb += BLOCK)
+      if (c.slice == 0) process_scalar(hb + tid, hb + tid < head);
+    for (int64_t tb = tail0; tb < c.len; tb += BLOCK)
+      if (c.slice == c.nslices - 1) process_scalar(tb + tid, tb + tid < c.len);
+  } else {
+    // ---- source = candidate buffer written by the previous pass (codes + indices) ----
+    const unsigned long long n = c.nbuf;
+    const unsigned long long per = (n + c.nslices - 1) / c.nslices;
+    const unsigned long long e0 = std::min<unsigned long long>(n, (unsigned long long)c.slice * per);
+    const unsigned long long e1 = std::min<unsigned long long>(n, e0 + per);
+    nread = n;
+    if constexpr (DF != 0) {
+      for (unsigned long long base = e0; base < e1; base += BLOCK) {
+        const unsigned long long i = base + tid;
+        const bool valid = i < e1;
+        const U code = valid ? c.bcin[i] : (U)0;
+        const IdxT idx = valid ? c.biin[i] : (IdxT)0;
+        bool win, cand;
+        classify(code, idx, valid, win, cand);
+        if (do_hist && cand) hist_cand(code, idx);
+        push_out(win, code, idx);
+        if (store) push_buf(cand, code, idx);
+      }
+    }
+  }
+  if constexpr (DF != 0) {
+    __syncwarp();
+    if (ocnt) wq_flush<KIND, IdxT>(c.oq, ocnt, c.outc, c.kk, c.ov, c.oi, 0, sel_min, c.err);
+    if (bcnt) wq_flush<KIND, IdxT>(c.bq, bcnt, c.bufc, c.capa, c.bco, c.bio, 1, sel_min, c.err);
+  }
+  return nread;
+}
+
+}  // namespace airtopk

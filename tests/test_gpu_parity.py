@@ -235,3 +235,31 @@ def test_repeated_calls_reuse_workspace():
         v, i = at.select(xd, 300, workspace=ws)
     torch.cuda.synchronize()
     assert_parity(x, "f32", 300, True, to_bits(v, "f32"), i.cpu().numpy())
+
+
+# ---------------------------------------------------------------- both engines, every cluster size
+
+@pytest.mark.parametrize("engine,cs", [(1, 0), (2, 1), (2, 2), (2, 4), (2, 8), (2, 16)])
+@pytest.mark.parametrize("dist,batch,n,k", [("normal", 37, 1 << 16, 256), ("uniform", 3, 300001, 5000),
+                                            ("adversarial", 5, 1 << 18, 20000), ("uniform", 1, 1 << 16, 32)])
+def test_engines(engine, cs, dist, batch, n, k):
+    x = _keys(dist, 61, batch, n)
+    for sm in (True, False):
+        v, i = gpu_select(x, "f32", k, sm, engine=engine, cluster_size=cs)
+        assert_parity(x, "f32", k, sm, v, i)
+
+
+@pytest.mark.parametrize("dtn", ["f16", "bf16", "f64", "u32"])
+def test_cluster_engine_dtypes(dtn):
+    u = gen.u64(91, 8 * 20011)
+    raw = u.astype({"f16": np.uint16, "bf16": np.uint16, "f64": np.uint64, "u32": np.uint32}[dtn]).reshape(8, 20011)
+    for k in (1, 500, 20010):
+        v, i = gpu_select(raw, dtn, k, True, engine=2)
+        assert_parity(raw, dtn, k, True, v, i)
+
+
+@pytest.mark.parametrize("alpha", [1, 128, 1 << 40])
+def test_cluster_engine_alpha(alpha):
+    x = _keys("adversarial", 13, 6, 1 << 17, 10)
+    v, i = gpu_select(x, "f32", 3000, alpha=alpha, engine=2)
+    assert_parity(x, "f32", 3000, True, v, i)

@@ -1,0 +1,152 @@
+// microbench_hist.cu — pass-1 histogram strategies on B200 (2048 bins of the top 11 key bits).
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o microbench_hist tools/microbench_hist.cu
+// Prints GB/s of one read of 2^30 f32 keys per strategy and data distribution.
+#include <cstdio>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+constexpr int kBins = 2048;
+
+__device__ __forceinline__ uint64_t mix64(uint64_t z) {
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+  return z ^ (z >> 31);
+}
+
+__global__ void fill(float* x, int64_t n, int dist) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t u = (uint32_t)(mix64(12345 + (i + 1) * 0x9E3779B97F4A7C15ULL) >> 32);
+    float f;
+    if (dist == 0) f = (float)u * 2.3283064365386963e-10f + 1.1641532182693481e-10f;
+    else if (dist == 1) { uint32_t b = 0x3F800000u | (u & 0xFFFu); f = __uint_as_float(b); }
+    else { uint32_t b = 0x3F800000u | (u & 0xFFFFFu); f = __uint_as_float(b); }  // M=12
+    x[i] = f;
+  }
+}
+
+__device__ __forceinline__ uint4 ldg_stream(const uint4* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+
+__device__ __forceinline__ uint32_t code_of(uint32_t b) { return b ^ ((uint32_t)((int32_t)b >> 31) | 0x80000000u); }
+
+template <int MODE, int R>
+__device__ __forceinline__ void add(uint32_t* sh, uint32_t d, int lane, uint32_t& cur, uint32_t& cnt) {
+  if (MODE == 1) {
+    atomicAdd(&sh[d], 1u);
+  } else if (MODE == 2) {  // R copies, copy chosen by lane
+    atomicAdd(&sh[d * R + (lane % R)], 1u);
+  } else if (MODE == 3) {  // match_any
+    unsigned g = __match_any_sync(0xffffffffu, d);
+    if (lane == __ffs(g) - 1) atomicAdd(&sh[d], (unsigned)__popc(g));
+  } else if (MODE == 4) {  // thread-local run length + R copies
+    if (d == cur) ++cnt;
+    else {
+      if (cnt) atomicAdd(&sh[cur * R + (lane % R)], cnt);
+      cur = d; cnt = 1;
+    }
+  }
+}
+
+template <int MODE, int R, int UNROLL>
+__global__ void __launch_bounds__(512) hist(const float* x, int64_t n, uint32_t* out, uint32_t* sink) {
+  extern __shared__ uint32_t sh[];
+  const int nb = (MODE == 2 || MODE == 4) ? kBins * R : kBins;
+  for (int i = threadIdx.x; i < nb; i += blockDim.x) sh[i] = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t nvec = n / 4;
+  const int64_t per = (nvec + gridDim.x - 1) / gridDim.x;
+  const int64_t v0 = blockIdx.x * per, v1 = min(nvec, v0 + per);
+  const uint4* vp = (const uint4*)x;
+  uint32_t acc = 0, cur = 0xffffffffu, cnt = 0;
+  int64_t base = v0;
+  for (; base + (int64_t)UNROLL * 512 <= v1; base += (int64_t)UNROLL * 512) {
+    uint4 r[UNROLL];
+#pragma unroll
+    for (int u = 0; u < UNROLL; ++u) r[u] = ldg_stream(vp + base + u * 512 + threadIdx.x);
+#pragma unroll
+    for (int u = 0; u < UNROLL; ++u) {
+      uint32_t e[4] = {r[u].x, r[u].y, r[u].z, r[u].w};
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        uint32_t d = code_of(e[j]) >> 21;
+        if (MODE == 0) acc += d;
+        else add<MODE, R>(sh, d, lane, cur, cnt);
+      }
+    }
+  }
+  for (int64_t v = base + threadIdx.x; v < v1; v += 512) {
+    uint4 q = ldg_stream(vp + v);
+    uint32_t e[4] = {q.x, q.y, q.z, q.w};
+    for (int j = 0; j < 4; ++j) {
+      uint32_t d = code_of(e[j]) >> 21;
+      if (MODE == 0) acc += d;
+      else if (MODE == 4) { if (d == cur) ++cnt; else { if (cnt) atomicAdd(&sh[cur * R + (lane % R)], cnt); cur = d; cnt = 1; } }
+      else if (MODE == 3) atomicAdd(&sh[d], 1u);
+      else if (MODE == 2) atomicAdd(&sh[d * R + (lane % R)], 1u);
+      else atomicAdd(&sh[d], 1u);
+    }
+  }
+  if (MODE == 4 && cnt) atomicAdd(&sh[cur * R + (lane % R)], cnt);
+  __syncthreads();
+  if (MODE == 0) { if (acc == 0x12345678u) sink[0] = acc; return; }
+  for (int b = threadIdx.x; b < kBins; b += blockDim.x) {
+    uint32_t s = 0;
+    if (MODE == 2 || MODE == 4) { for (int c = 0; c < R; ++c) s += sh[b * R + c]; }
+    else s = sh[b];
+    if (s) atomicAdd(&out[b], s);
+  }
+}
+
+template <int MODE, int R, int UNROLL>
+void run(const char* name, const float* x, int64_t n, uint32_t* out, uint32_t* sink, int blocks_per_sm) {
+  const int nb = (MODE == 2 || MODE == 4) ? kBins * R : kBins;
+  size_t smem = nb * 4;
+  cudaFuncSetAttribute(hist<MODE, R, UNROLL>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  int occ = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, hist<MODE, R, UNROLL>, 512, smem);
+  int grid = 148 * (blocks_per_sm ? blocks_per_sm : occ);
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  for (int w = 0; w < 3; ++w) hist<MODE, R, UNROLL><<<grid, 512, smem>>>(x, n, out, sink);
+  cudaEventRecord(a);
+  const int it = 10;
+  for (int w = 0; w < it; ++w) hist<MODE, R, UNROLL><<<grid, 512, smem>>>(x, n, out, sink);
+  cudaEventRecord(b);
+  cudaEventSynchronize(b);
+  float ms;
+  cudaEventElapsedTime(&ms, a, b);
+  ms /= it;
+  printf("%-28s occ=%d grid=%d  %.3f ms  %.0f GB/s\n", name, occ, grid, ms, n * 4.0 / (ms * 1e-3) / 1e9);
+}
+
+int main() {
+  const int64_t n = 1LL << 30;
+  float* x;
+  uint32_t *out, *sink;
+  cudaMalloc(&x, n * 4);
+  cudaMalloc(&out, kBins * 4);
+  cudaMalloc(&sink, 4);
+  const char* dn[3] = {"uniform", "adversarial M=20", "adversarial M=12"};
+  for (int dist = 0; dist < 3; ++dist) {
+    fill<<<148 * 8, 512>>>(x, n, dist);
+    cudaDeviceSynchronize();
+    printf("== %s\n", dn[dist]);
+    run<0, 1, 4>("load-only", x, n, out, sink, 0);
+    run<0, 1, 8>("load-only u8", x, n, out, sink, 0);
+    run<1, 1, 4>("plain atomics", x, n, out, sink, 0);
+    run<2, 4, 4>("R=4 copies", x, n, out, sink, 0);
+    run<2, 8, 4>("R=8 copies", x, n, out, sink, 0);
+    run<2, 16, 4>("R=16 copies", x, n, out, sink, 0);
+    run<3, 1, 4>("match_any", x, n, out, sink, 0);
+    run<4, 1, 4>("RLE + 1 copy", x, n, out, sink, 0);
+    run<4, 8, 4>("RLE + 8 copies", x, n, out, sink, 0);
+  }
+  cudaError_t e = cudaGetLastError();
+  printf("err=%s\n", cudaGetErrorString(e));
+  return 0;
+}
