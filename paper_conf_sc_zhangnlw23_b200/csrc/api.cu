@@ -83,7 +83,7 @@ Plan make_plan(const SelectArgs& a) {
 // and small rows, the grid engine (one launch per pass, whole GPU per row) for long rows.
 static int auto_engine(const SelectArgs& a) {
   if (a.len <= (int64_t(1) << 17)) return 2;
-  if (a.len <= (int64_t(1) << 22) && a.batch >= 16) return 2;
+  if (a.len <= (int64_t(1) << 22) && a.batch >= 16 && getenv("AIRTOPK_CLUSTER_BATCHED")) return 2;
   return 1;
 }
 

@@ -12,6 +12,7 @@
 #pragma once
 
 #include <cstdint>
+#include <type_traits>
 #include <cuda_runtime.h>
 
 namespace airtopk {
@@ -45,6 +46,22 @@ __device__ __forceinline__ typename KT<KIND>::U to_code(typename KT<KIND>::U b, 
     c = b;
   }
   return sel_min ? c : U(~c);
+}
+
+// Branch-free form of to_code for the streaming loops: xmask = 0 (select-min) or all ones
+// (select-max). b ^ (sign-extended sign | sign bit): flips every bit of negatives, sets the sign bit of
+// non-negatives.
+template <int KIND>
+__device__ __forceinline__ typename KT<KIND>::U to_code_x(typename KT<KIND>::U b, typename KT<KIND>::U xmask) {
+  using U = typename KT<KIND>::U;
+  if constexpr (KT<KIND>::IEEE) {
+    using S = std::make_signed_t<U>;
+    constexpr U sign = U(U(1) << (KT<KIND>::R - 1));
+    const U m = (U)((S)b >> (KT<KIND>::R - 1));
+    return U(b ^ (m | sign) ^ xmask);
+  } else {
+    return U(b ^ xmask);
+  }
 }
 
 template <int KIND>

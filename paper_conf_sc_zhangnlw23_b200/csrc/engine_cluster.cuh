@@ -124,7 +124,7 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
       c.bq = &sh_bq[warp];
       const bool hist_on = c.do_hist || DF == 0;
       if (hist_on) {
-        for (int i = tid; i < kMaxBins * HC; i += kCBlock) sh_hist[i] = 0;
+        for (int i = tid; i < kHistSlots * HC; i += kCBlock) sh_hist[i] = 0;
       }
       __syncthreads();
       switch (DF * 3 + DH) {
@@ -209,7 +209,7 @@ namespace airtopk {
 template <int KIND, typename IdxT, bool HASIDX>
 cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t s) {
   auto kern = cluster_kernel<KIND, IdxT, HASIDX>;
-  constexpr size_t smem = (size_t)kMaxBins * 4 * hist_copies<KIND, IdxT, 1>();
+  constexpr size_t smem = (size_t)kHistSlots * 4 * hist_copies<KIND, IdxT, 1>();
   static const cudaError_t attr1 = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   static const cudaError_t attr2 = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
   if (attr1 != cudaSuccess) return attr1;

@@ -128,7 +128,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pass_kernel(const GridPara
 
   const bool hist_on = c.do_hist || DF == 0;
   if (hist_on) {
-    for (int i = tid; i < kMaxBins * HC; i += kBlock) sh_hist[i] = 0;
+    for (int i = tid; i < kHistSlots * HC; i += kBlock) sh_hist[i] = 0;
     __syncthreads();
   }
 
@@ -192,7 +192,7 @@ struct Events {
 
 template <int KIND, typename IdxT, int DF, int DH>
 constexpr size_t hist_smem_bytes() {
-  return (size_t)kMaxBins * 4 * hist_copies<KIND, IdxT, DF>();
+  return (size_t)kHistSlots * 4 * hist_copies<KIND, IdxT, DF>();
 }
 
 template <int KIND, typename IdxT, int DF, int DH, bool HASIDX>

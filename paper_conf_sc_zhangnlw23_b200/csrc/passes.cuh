@@ -28,6 +28,15 @@ constexpr int kQCap = 64;
 // (interleaved bin-major so copies of one bin sit in different banks); cuts the same-address
 // serialisation of shared atomics when many lanes hit a few bins (radix-adversarial passes).
 constexpr int kHistCopies = 4;
+// Extra histogram slot that absorbs the atomics of non-candidates / invalid lanes (never scanned).
+constexpr int kDummyBin = kMaxBins;
+constexpr int kHistSlots = kMaxBins + 32;  // per copy; the dummy bin + padding
+
+// +1 on a shared-window address (no return value): red.shared.add, which the hardware aggregates
+// over lanes hitting the same address.
+__device__ __forceinline__ void shared_inc(unsigned addr) {
+  asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(addr) : "memory");
+}
 
 template <typename U, typename IdxT>
 struct WarpQ {
@@ -148,7 +157,19 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
     ti = (IdxT)(c.tidx >> sf);
     bi = ti & ~(IdxT)((1u << c.df.width) - 1u);
   }
-  unsigned* const hist_lane = c.hist + (HC > 1 ? (lane % HC) : 0);
+  // Fast classification for adjacent key digits (DF == 1, DH == 1, sf == shh + w): with
+  // t = code >> shh and B = bc << w, y = t - B lies in [0, S) for results (higher digits == prefix,
+  // digit q-1 < j), in [S, S + nb) for candidates (x = y - S is then digit q), and >= S + nb (or
+  // wraps) otherwise. S = (tc - bc) << w, nb = 2^w.
+  const int wq_ = c.dh.width;
+  const W kx_B = (DF == 1) ? (W)(bc << wq_) : (W)0;
+  const W kx_S = (DF == 1) ? (W)((tc - bc) << wq_) : (W)0;
+  const W kx_nb = (W)1 << wq_;
+  const W kx_Swin = kx_S + (emit_all ? kx_nb : (W)0);
+  const W kx_nbS = store ? kx_nb : (W)0;
+  // shared-window address of this lane's histogram copy (c.hist is the dynamic smem base)
+  const unsigned hbase = (unsigned)__cvta_generic_to_shared(c.hist) + ((HC > 1) ? (unsigned)(lane % HC) * 4u : 0u);
+  const U xmask = sel_min ? (U)0 : (U)~(U)0;
   int ocnt = 0, bcnt = 0;
 
   auto push_out = [&](bool pred, U code, IdxT idx) {
@@ -167,17 +188,21 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
     } else {
       const bool ce = (code == fc);
       const IdxT h = (IdxT)(idx >> sf);
-      lt = ce & ((IdxT)(h - bi) < (IdxT)(ti - bi));
-      eq = ce & (h == ti);
+      lt = ce && ((IdxT)(h - bi) < (IdxT)(ti - bi));
+      eq = ce && (h == ti);
     }
-    win = valid & (lt | (emit_all & eq));
-    cand = valid & !emit_all & eq;
+    win = valid && (lt || (emit_all && eq));
+    cand = valid && !emit_all && eq;
   };
-  auto hist_cand = [&](U code, IdxT idx) {  // Alg1 L19-20
+  // Alg1 L19-20. Non-candidates count into a dummy bin instead of branching: a warp-uniform address
+  // is aggregated by the shared atomic unit (ATOMS.POPC.INC), so the common "no candidate" case is
+  // one cheap atomic and no divergence.
+  auto hist_cand = [&](U code, IdxT idx, bool cand) {
     unsigned d;
     if constexpr (DH == 2) d = (unsigned)(idx >> shh) & hmask;
     else d = (unsigned)((W)code >> shh) & hmask;
-    atomicAdd(&hist_lane[d * HC], 1u);
+    d = (cand && do_hist) ? d : (unsigned)kDummyBin;
+    shared_inc(hbase + d * (HC * 4));
   };
 
   unsigned long long nread;
@@ -199,26 +224,50 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
       else return (IdxT)pos;
     };
 
-    auto process_tile = [&](const uint4 (&r)[kUnroll], int64_t vb, int64_t vlim) {
+    // One thread's tile: kUnroll 16-byte vectors at vector indices vb + u*BLOCK. FULL: all valid.
+    auto process_tile = [&](const uint4 (&r)[kUnroll], int64_t vb, int64_t vlim, auto full_tag) {
+      constexpr bool FULL = decltype(full_tag)::value;
       if constexpr (DF == 0) {
+        // pass 1: the top digit needs no mask (code >> shh < 2^11)
 #pragma unroll
         for (int u = 0; u < kUnroll; ++u) {
-          const bool valid = vb + (int64_t)u * BLOCK < vlim;
+          const bool valid = FULL || (vb + (int64_t)u * BLOCK < vlim);
 #pragma unroll
           for (int e = 0; e < VEC; ++e) {
-            const U code = to_code<KIND>(vec_elem<U>(r[u], e), sel_min);
-            if (valid) atomicAdd(&c.hist[((W)code >> shh) & hmask], 1u);
+            const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
+            const unsigned d = (unsigned)((W)code >> shh);
+            shared_inc(hbase + 4u * (valid ? d : (unsigned)kDummyBin));
+          }
+        }
+        return;
+      }
+      unsigned fl = 0;  // elements that must leave through the queues (results / stored candidates)
+      if constexpr (DF == 1 && DH == 1) {
+        // adjacent key digits: y = (code >> shh) - B places the elements whose higher digits match
+        // the prefix at [S, S + nb) and the results below S (see the derivation at kx_* below)
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+          const bool valid = FULL || (vb + (int64_t)u * BLOCK < vlim);
+#pragma unroll
+          for (int e = 0; e < VEC; ++e) {
+            const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
+            const W y = ((W)code >> shh) - kx_B;
+            const W x = y - kx_S;
+            const bool win = y < kx_Swin;
+            const bool cst = x < kx_nbS;
+            const unsigned d = (unsigned)min(x, (W)kDummyBin);
+            shared_inc(hbase + (valid ? d : (unsigned)kDummyBin) * (HC * 4u));
+            if (valid && (win || cst)) fl |= 1u << (u * VEC + e);
           }
         }
       } else {
-        unsigned fw = 0, fcand = 0;  // per-element result / stored-candidate flags
 #pragma unroll
         for (int u = 0; u < kUnroll; ++u) {
           const int64_t v = vb + (int64_t)u * BLOCK;
-          const bool valid = v < vlim;
+          const bool valid = FULL || (v < vlim);
 #pragma unroll
           for (int e = 0; e < VEC; ++e) {
-            const U code = to_code<KIND>(vec_elem<U>(r[u], e), sel_min);
+            const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
             IdxT idx = 0;
             if constexpr (DF == 2 || DH == 2) {
               // the index is needed to classify (DF == 2) or to histogram a candidate (DH == 2)
@@ -228,25 +277,25 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
             }
             bool win, cand;
             classify(code, idx, valid, win, cand);
-            if (do_hist && cand) hist_cand(code, idx);
-            fw |= (unsigned)win << (u * VEC + e);
-            fcand |= (unsigned)(cand & store) << (u * VEC + e);
+            hist_cand(code, idx, cand);
+            if (win || (cand && store)) fl |= 1u << (u * VEC + e);
           }
         }
-        // slow path (rare in most passes): results / candidates through the warp queues
-        unsigned fl = fw | fcand;
-        while (__any_sync(kFull, fl != 0)) {
-          const int b = fl ? __ffs(fl) - 1 : 0;
-          const bool w = (fw >> b) & (fl != 0), cd = (fcand >> b) & (fl != 0);
-          fl &= fl - 1;
-          // re-read the flagged element (an L2 hit: this warp just streamed it) instead of keeping
-          // the tile registers alive across the slow path
-          const int64_t pos = head + (vb + (int64_t)(b / VEC) * BLOCK) * VEC + (b % VEC);
-          const U code = to_code<KIND>((w | cd) ? __ldcg(rowp + pos) : (U)0, sel_min);
-          const IdxT idx = (w | cd) ? index_of(pos) : (IdxT)0;
-          push_out(w, code, idx);
-          if (store) push_buf(cd, code, idx);
-        }
+      }
+      // slow path (rare in most passes): results / candidates through the warp queues. The flagged
+      // element is re-read (an L2 hit: this warp just streamed it) and re-classified, so the tile
+      // registers die early.
+      while (__any_sync(kFull, fl != 0)) {
+        const bool has = fl != 0;
+        const int b = has ? __ffs(fl) - 1 : 0;
+        fl &= fl - 1;
+        const int64_t pos = head + (vb + (int64_t)(b / VEC) * BLOCK) * VEC + (b % VEC);
+        const U code = to_code_x<KIND>(has ? __ldcg(rowp + pos) : (U)0, xmask);
+        const IdxT idx = has ? index_of(pos) : (IdxT)0;
+        bool w, cd;
+        classify(code, idx, has, w, cd);
+        push_out(w, code, idx);
+        if (store) push_buf(cd, code, idx);
       }
     };
 
@@ -258,7 +307,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
       uint4 r[kUnroll];
 #pragma unroll
       for (int u = 0; u < kUnroll; ++u) r[u] = ldg_stream(vp + vb + (int64_t)u * BLOCK);
-      process_tile(r, vb, v1);
+      process_tile(r, vb, v1, std::true_type{});
     }
     if (v0 + nfull * tile < v1) {
       const int64_t vb = v0 + nfull * tile + tid;
@@ -268,18 +317,18 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
         const int64_t v = vb + (int64_t)u * BLOCK;
         r[u] = (v < v1) ? ldg_stream(vp + v) : make_uint4(0, 0, 0, 0);
       }
-      process_tile(r, vb, v1);
+      process_tile(r, vb, v1, std::false_type{});
     }
     // scalar head (slice 0) and tail (last slice) of a misaligned / ragged row
     auto process_scalar = [&](int64_t i, bool valid) {
       const U code = to_code<KIND>(valid ? rowp[i] : (U)0, sel_min);
       if constexpr (DF == 0) {
-        if (valid) atomicAdd(&c.hist[((W)code >> shh) & hmask], 1u);
+        shared_inc(hbase + 4u * (valid ? (unsigned)(((W)code >> shh) & hmask) : (unsigned)kDummyBin));
       } else {
         const IdxT idx = valid ? index_of(i) : (IdxT)0;
         bool win, cand;
         classify(code, idx, valid, win, cand);
-        if (do_hist && cand) hist_cand(code, idx);
+        hist_cand(code, idx, cand);
         push_out(win, code, idx);
         if (store) push_buf(cand, code, idx);
       }
@@ -303,7 +352,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
         const IdxT idx = valid ? c.biin[i] : (IdxT)0;
         bool win, cand;
         classify(code, idx, valid, win, cand);
-        if (do_hist && cand) hist_cand(code, idx);
+        hist_cand(code, idx, cand);
         push_out(win, code, idx);
         if (store) push_buf(cand, code, idx);
       }
