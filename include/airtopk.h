@@ -96,8 +96,11 @@ typedef struct {
                            Grid engine only. NULL = no trace. */
   void* const* events;  /* optional array of n_events cudaEvent_t (created by the caller) recorded on
                            `stream` around the launches: events[0] before the first kernel,
-                           events[q+1] after launch q — lets a caller time each kernel with CUDA
+                           events[i+1] after launch i — lets a caller time each kernel with CUDA
                            events on the launching stream. NULL = none. */
+  int32_t window;       /* sample-guided window pass: 0 = auto (grid engine,
+                           len >= 2^18), 1 = on, -1 = off (the paper's passes only). Exact either way. */
+  int32_t reserved1;
 } airtopk_options;
 
 #define AIRTOPK_TRACE_MAX_PASSES 16
@@ -149,6 +152,22 @@ airtopk_status airtopk_select_with_idx(const void* keys, const int64_t* in_idx, 
 airtopk_status airtopk_select_host(const void* h_keys, airtopk_dtype dtype, int64_t batch, int64_t len,
                                    int64_t k, int select_min, void* h_out_vals, int64_t* h_out_idx,
                                    airtopk_stream_t stream);
+
+/* How a call with these arguments would run (no device work; may query the current device's SM
+ * count). Lets callers count launches and label measurements. */
+typedef struct {
+  int32_t engine;        /* airtopk_engine actually used (3 = K == len trivial copy) */
+  int32_t passes;        /* radix passes P (key digits + index digits) */
+  int32_t launches;      /* kernel launches per call, excluding the workspace memset */
+  int32_t ctas_per_row;  /* grid engine */
+  int32_t cluster_size;  /* cluster engine */
+  int32_t index_bits;    /* bits of the row index appended for the lowest-index tie-break */
+  int64_t buffer_cap;    /* candidate-buffer capacity per row (floor((len-1)/alpha)) */
+  size_t workspace_bytes;
+} airtopk_plan;
+
+airtopk_status airtopk_describe(airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k,
+                                const airtopk_options* opt, airtopk_plan* out);
 
 /* Human-readable status; never NULL. */
 const char* airtopk_status_str(airtopk_status s);

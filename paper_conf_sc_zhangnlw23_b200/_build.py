@@ -5,6 +5,7 @@
 from __future__ import annotations
 
 import glob
+import hashlib
 import os
 import subprocess
 import sys
@@ -12,7 +13,8 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-LIB = os.path.join(PKG, "libairtopk.so")
+LIB = os.environ.get("AIRTOPK_LIB_OUT", os.path.join(PKG, "libairtopk.so"))
+EXTRA = os.environ.get("AIRTOPK_NVCC_FLAGS", "").split()
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -41,9 +43,10 @@ def build(force: bool = False, verbose: bool = False) -> str:
     os.makedirs(os.path.join(PKG, "build"), exist_ok=True)
     procs = []
     for src in sources():
-        obj = os.path.join(PKG, "build", os.path.basename(src) + ".o")
+        tag = ("." + hashlib.md5(" ".join(EXTRA).encode()).hexdigest()[:8]) if EXTRA else ""
+        obj = os.path.join(PKG, "build", os.path.basename(src) + tag + ".o")
         cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3",
-               "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]
+               "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include"), *EXTRA, "-c", src, "-o", obj]
         if verbose:
             cmd += ["-Xptxas", "-v"]
         procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))

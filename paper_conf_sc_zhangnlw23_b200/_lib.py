@@ -8,7 +8,7 @@ import ctypes
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libairtopk.so")
+LIB_PATH = os.environ.get("AIRTOPK_LIB", os.path.join(_PKG, "libairtopk.so"))
 
 OK, EINVAL, EDTYPE, ENOSPACE, ECUDA = 0, 1, 2, 3, 4
 F32, F16, BF16, F64, U32 = 0, 1, 2, 3, 4
@@ -22,6 +22,7 @@ EXPORTS = (
     "airtopk_select_f32", "airtopk_select_f16", "airtopk_select_bf16", "airtopk_select_f64",
     "airtopk_select_u32", "airtopk_workspace_bytes_with_idx", "airtopk_select_with_idx",
     "airtopk_select_host", "airtopk_status_str", "airtopk_last_cuda_error", "airtopk_version",
+    "airtopk_describe",
 )
 
 
@@ -34,6 +35,21 @@ class Options(ctypes.Structure):
         ("n_events", ctypes.c_int32),
         ("trace", ctypes.c_void_p),
         ("events", ctypes.c_void_p),
+        ("window", ctypes.c_int32),
+        ("reserved1", ctypes.c_int32),
+    ]
+
+
+class Plan(ctypes.Structure):
+    _fields_ = [
+        ("engine", ctypes.c_int32),
+        ("passes", ctypes.c_int32),
+        ("launches", ctypes.c_int32),
+        ("ctas_per_row", ctypes.c_int32),
+        ("cluster_size", ctypes.c_int32),
+        ("index_bits", ctypes.c_int32),
+        ("buffer_cap", ctypes.c_int64),
+        ("workspace_bytes", ctypes.c_size_t),
     ]
 
 
@@ -74,4 +90,6 @@ def load(path: str = LIB_PATH):
     lib.airtopk_status_str.restype = ctypes.c_char_p
     lib.airtopk_last_cuda_error.restype = ci
     lib.airtopk_version.restype = ctypes.c_char_p
+    lib.airtopk_describe.argtypes = [ci, i64, i64, i64, ctypes.POINTER(Options), ctypes.POINTER(Plan)]
+    lib.airtopk_describe.restype = ci
     return lib

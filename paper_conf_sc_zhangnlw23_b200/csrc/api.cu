@@ -75,7 +75,14 @@ Plan make_plan(const SelectArgs& a) {
   p.off_hist = align_up(sizeof(RowState) * (size_t)a.batch, 256);
   p.off_bcode = p.off_hist + align_up((size_t)a.batch * 2 * kMaxBins * csz, 256);
   p.off_bidx = p.off_bcode + align_up((size_t)2 * a.batch * p.cap_alloc * key_bytes(a.kind), 256);
-  p.bytes = p.off_bidx + align_up((size_t)2 * a.batch * p.cap_alloc * isz, 256);
+  // sample-guided window (grid engine, position indices): ~len/256 stratified samples, 1K..16K
+  p.nsamp = 0;
+  if (!a.in_idx && (a.window > 0 || (a.window == 0 && a.len >= (int64_t(1) << 18)))) {
+    int64_t ns = std::min<int64_t>(std::max<int64_t>(a.len / 256, 1024), 16384);
+    p.nsamp = (int)std::min<int64_t>(ns, a.len);
+  }
+  p.off_samp = p.off_bidx + align_up((size_t)2 * a.batch * p.cap_alloc * isz, 256);
+  p.bytes = p.off_samp + align_up((size_t)a.batch * p.nsamp * (key_bytes(a.kind) == 8 ? 8 : 4), 256);
   return p;
 }
 
@@ -109,7 +116,8 @@ static void choose_launch(const SelectArgs& a, Plan& p) {
   const int64_t target = (int64_t)num_sms() * grid_blocks_per_sm(a, p.idx64);
   const int64_t chunk = grid_vec_chunk(a.kind);
   const int64_t maxc = std::max<int64_t>(1, (a.len + chunk - 1) / chunk);
-  int64_t c = (target + a.batch - 1) / a.batch;
+  // whole waves: batch x cpr <= target CTAs (a partial second wave costs more than idle slots)
+  int64_t c = std::max<int64_t>(1, target / a.batch);
   p.cpr = (int)std::max<int64_t>(1, std::min<int64_t>(c, maxc));
 }
 
@@ -121,6 +129,7 @@ static airtopk_status validate(const SelectArgs& a) {
   if (a.batch < 1 || a.len < 1 || a.k < 1 || a.k > a.len) return AIRTOPK_EINVAL;
   if (a.alpha < 0) return AIRTOPK_EINVAL;
   if (a.engine < 0 || a.engine > 2) return AIRTOPK_EINVAL;
+  if (a.window < -1 || a.window > 1) return AIRTOPK_EINVAL;
   if (a.in_idx && (a.batch != 1 || a.idx_bits < 1 || a.idx_bits > 63)) return AIRTOPK_EINVAL;
   return AIRTOPK_OK;
 }
@@ -165,6 +174,7 @@ static SelectArgs make_args(const void* keys, int dt, int64_t batch, int64_t len
     a.trace = opt->trace;
     a.events = opt->events;
     a.n_events = opt->events ? opt->n_events : 0;
+    a.window = opt->window;
   }
   if (a.alpha == 0) a.alpha = 128;
   return a;
@@ -283,6 +293,28 @@ airtopk_status airtopk_select_host(const void* h_keys, airtopk_dtype dtype, int6
   cudaFreeAsync(d, s);
   if ((e = cudaStreamSynchronize(s)) != cudaSuccess && st == AIRTOPK_OK) st = fail_cuda(e);
   return st;
+}
+
+airtopk_status airtopk_describe(airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k,
+                                const airtopk_options* opt, airtopk_plan* out) {
+  if (!out) return AIRTOPK_EINVAL;
+  int64_t dummy = 0;
+  SelectArgs a = make_args((const void*)1, (int)dtype, batch, len, k, 1, (void*)1, &dummy, opt);
+  airtopk_status st = validate(a);
+  if (st != AIRTOPK_OK) return st;
+  Plan p = make_plan(a);
+  const size_t bytes = p.engine == 3 ? 0 : p.bytes;
+  choose_launch(a, p);
+  std::memset(out, 0, sizeof(*out));
+  out->engine = p.engine;
+  out->passes = p.P;
+  out->launches = p.engine == 3 ? 1 : (p.engine == 2 ? 1 : p.P + 1 + (p.nsamp > 0 ? 2 : 0));
+  out->ctas_per_row = p.engine == 1 ? p.cpr : 0;
+  out->cluster_size = p.engine == 2 ? p.csize : 0;
+  out->index_bits = p.IB;
+  out->buffer_cap = p.cap_rule;
+  out->workspace_bytes = bytes;
+  return AIRTOPK_OK;
 }
 
 const char* airtopk_status_str(airtopk_status s) {

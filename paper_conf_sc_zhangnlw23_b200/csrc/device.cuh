@@ -113,6 +113,9 @@ struct alignas(128) RowState {
   int stop1;                     // 1 + pass after whose scan K == C (early stop); 0 = none
   unsigned int j;
   unsigned int error;            // 1 = output overflow (duplicate in_idx), 2 = buffer overflow
+  int src1;                      // source of the next pass: 0 = input row L, s + 1 = buffer slot s
+  int win_state;                 // sample-guided window: 0 off, 1 window holds the K-th key, 2 failed
+  unsigned long long win_lo, win_hi;  // window [lo, hi] of codes chosen from the sample
 };
 
 template <typename T>
@@ -145,6 +148,11 @@ __device__ __forceinline__ unsigned long long warp_alloc(bool pred, unsigned lon
   }
   return base + __popc(mask & lanemask_lt());
 }
+
+// Programmatic dependent launch (PDL): wait for the previous kernel in the stream (its writes are
+// then visible), and let the next kernel's CTAs be scheduled as ours retire. No-ops without PDL.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
 // 128-bit streaming load of read-only input (no L1 allocation).
 __device__ __forceinline__ uint4 ldg_stream(const uint4* p) {

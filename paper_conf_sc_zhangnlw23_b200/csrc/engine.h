@@ -20,6 +20,7 @@ struct SelectArgs {
   int engine = 0;
   int ctas_per_row = 0;
   int cluster_size = 0;
+  int window = 0;                   // sample-guided window: 0 auto, 1 on, -1 off
   int64_t* trace = nullptr;
   void* const* events = nullptr;    // optional cudaEvent_t[n_events] recorded around launches
   int n_events = 0;
@@ -37,7 +38,8 @@ struct Plan {
   int cpr;           // CTAs per row (grid engine)
   int csize;         // CTAs per cluster (cluster engine)
   int max_clusters;  // cluster engine: clusters the workspace has candidate buffers for
-  size_t off_state, off_hist, off_bcode, off_bidx, bytes;
+  int nsamp;         // grid engine: samples per row for the sample-guided window (0 = off)
+  size_t off_state, off_hist, off_bcode, off_bidx, off_samp, bytes;
 };
 
 int key_bits(int kind);

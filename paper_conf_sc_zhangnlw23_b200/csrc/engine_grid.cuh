@@ -61,22 +61,28 @@ struct GridParams {
   int64_t cap_rule, cap_alloc;
   int cpr;
   int64_t* trace;
+  void* samp;  // sample-guided window: [batch][nsamp] sampled codes
 };
 
 constexpr int kBlock = 512;
 constexpr int kWarps = kBlock / 32;
 constexpr int kMinBlocks = 3;
+constexpr int kMinBlocksFilter = AIRTOPK_SLOW_REG ? 2 : 3;
 
+// Kernel q of the select. DF/DH: digit filtered / histogrammed (passes.cuh). DF == 3 is the
+// sample-guided window pass (q = 0); `redo` = the pass-0 histogram re-run over the window buffer.
 template <int KIND, typename IdxT, int DF, int DH, bool HASIDX>
-__global__ void __launch_bounds__(kBlock, kMinBlocks) pass_kernel(const GridParams p, const int q) {
+__global__ void __launch_bounds__(kBlock, (DF == 0 ? kMinBlocks : kMinBlocksFilter))
+    pass_kernel(const GridParams p, const int q, const int redo) {
   using U = typename KT<KIND>::U;
   using CountT = std::conditional_t<sizeof(IdxT) == 8, unsigned long long, unsigned>;
   constexpr bool HAS_Q = DF != 0;
+  constexpr bool FILTER = (DF == 1 || DF == 2);  // Alg1 L15-22 filter of digit q-1
   constexpr int HC = hist_copies<KIND, IdxT, DF>();
 
-  extern __shared__ unsigned sh_hist[];  // kMaxBins * HC counters (dynamic: may exceed 48 KB)
+  extern __shared__ unsigned sh_hist[];  // kHistSlots * HC counters (dynamic: may exceed 48 KB)
   __shared__ WarpQ<U, IdxT> sh_oq[HAS_Q ? kWarps : 1];
-  __shared__ WarpQ<U, IdxT> sh_bq[(HAS_Q && DH != 0) ? kWarps : 1];
+  __shared__ WarpQ<U, IdxT> sh_bq[(HAS_Q && (DH != 0 || DF == 3)) ? kWarps : 1];  // candidate queues
   __shared__ unsigned long long sh_tmp[kWarps];
   __shared__ ScanResult sh_res;
   __shared__ int sh_last;
@@ -86,45 +92,54 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pass_kernel(const GridPara
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
   RowState* st = p.st + row;
+  pdl_wait();     // the previous pass's scan (row state, buffers) is complete and visible
+  pdl_trigger();  // the next pass may be scheduled as our CTAs retire (hides launch latency)
 
   // ---- row state after scan q-1 ----
-  const int stop1 = (DF != 0) ? st->stop1 : 0;
-  if (DF != 0 && stop1 != 0 && stop1 - 1 < q - 1) return;  // finished by an earlier early stop
+  const int stop1 = FILTER ? st->stop1 : 0;
+  if (FILTER && stop1 != 0 && stop1 - 1 < q - 1) return;  // finished by an earlier early stop
+  const int win_state = (DF == 3 || (DF == 0 && redo)) ? st->win_state : 0;
+  if (DF == 3 && win_state != 1) return;                   // no window: pass 0 will read L
+  const bool redo_buf = (DF == 0) && redo && (win_state == 1);  // pass 0 over the window buffer
+  const int src1 = (FILTER || redo_buf) ? st->src1 : 0;    // Alg1 L7-8 (reading 6)
+  const int sslot = (src1 == 1) ? 1 : 0;                   // candidate buffer this pass writes
   PassCtx<U, IdxT> c;
   c.q = q;
-  c.emit_all = (DF != 0) && ((stop1 != 0 && stop1 - 1 == q - 1) || DH == 0);
+  c.emit_all = FILTER && ((stop1 != 0 && stop1 - 1 == q - 1) || DH == 0);
   c.do_hist = (DH != 0) && !c.emit_all;
-  const unsigned long long Cprev = (DF != 0) ? st->C : (unsigned long long)p.len;  // C_{q-1}
-  const unsigned long long Cpp = (DF != 0) ? st->Cp : (unsigned long long)p.len;   // C' = C_{q-2}
-  c.srcL = (DF == 0) || (Cpp > (unsigned long long)p.cap_rule);                   // Alg1 L7
-  c.store = c.do_hist && (DF != 0) && (Cprev <= (unsigned long long)p.cap_rule);  // Alg1 L17
+  const unsigned long long Cprev = (FILTER || redo_buf) ? st->C : (unsigned long long)p.len;  // C_{q-1}
+  c.srcL = (src1 == 0);
+  if (DF == 3) c.store = (win_state == 1);
+  else c.store = c.do_hist && FILTER && (Cprev <= (unsigned long long)p.cap_rule);  // Alg1 L17
   c.sel_min = p.sel_min != 0;
   c.reverse = (q & 1) != 0;  // walk back over what the previous pass left in L2
   c.dh = digit_of(q, KT<KIND>::R, p.IB);
-  c.df = digit_of(DF != 0 ? q - 1 : 0, KT<KIND>::R, p.IB);
-  c.tcode = (DF != 0) ? st->tcode : 0ull;
-  c.tidx = (DF != 0) ? st->tidx : 0ull;
+  c.df = digit_of(FILTER ? q - 1 : 0, KT<KIND>::R, p.IB);
+  c.tcode = FILTER ? st->tcode : 0ull;
+  c.tidx = FILTER ? st->tidx : 0ull;
+  c.lo = (win_state == 1) ? st->win_lo : 0ull;
+  c.span1 = (win_state == 1) ? st->win_hi - st->win_lo + 1ull : 0ull;
   c.rowp = (const U*)p.keys + row * p.len;
   c.rowi = HASIDX ? p.in_idx + row * p.len : nullptr;
   c.len = p.len;
   c.slice = cta;
   c.nslices = p.cpr;
-  const int islot = (q - 1) & 1;
+  const int islot = src1 > 0 ? src1 - 1 : 0;
   c.bcin = (const U*)p.bcode + ((size_t)islot * p.batch + row) * p.cap_alloc;
   c.biin = (const IdxT*)p.bidx + ((size_t)islot * p.batch + row) * p.cap_alloc;
-  c.nbuf = (DF != 0 && !c.srcL) ? st->buf_count[islot] : 0ull;
+  c.nbuf = (src1 > 0) ? st->buf_count[islot] : 0ull;
   c.ov = (U*)p.out_vals + row * p.k;
   c.oi = p.out_idx + row * p.k;
   c.outc = &st->out_count;
   c.kk = (unsigned long long)p.k;
-  c.bco = (U*)p.bcode + ((size_t)(q & 1) * p.batch + row) * p.cap_alloc;
-  c.bio = (IdxT*)p.bidx + ((size_t)(q & 1) * p.batch + row) * p.cap_alloc;
-  c.bufc = &st->buf_count[q & 1];
+  c.bco = (U*)p.bcode + ((size_t)sslot * p.batch + row) * p.cap_alloc;
+  c.bio = (IdxT*)p.bidx + ((size_t)sslot * p.batch + row) * p.cap_alloc;
+  c.bufc = &st->buf_count[sslot];
   c.capa = (unsigned long long)p.cap_alloc;
   c.err = &st->error;
   c.hist = sh_hist;
   c.oq = &sh_oq[HAS_Q ? warp : 0];
-  c.bq = &sh_bq[(HAS_Q && DH != 0) ? warp : 0];
+  c.bq = &sh_bq[(HAS_Q && (DH != 0 || DF == 3)) ? warp : 0];
 
   const bool hist_on = c.do_hist || DF == 0;
   if (hist_on) {
@@ -133,6 +148,33 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pass_kernel(const GridPara
   }
 
   const unsigned long long nread = run_pass<KIND, IdxT, DF, DH, HASIDX, kBlock>(c);
+
+  if constexpr (DF == 3) {
+    // ---- window pass: the last CTA validates the window. R results below lo, Wn members inside;
+    // the K-th key lies in the window iff R < K <= R + Wn (and the buffer did not overflow) ----
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) sh_last = (atomicAdd(&st->ticket, 1u) == (unsigned)(p.cpr - 1));
+    __syncthreads();
+    if (!sh_last || tid != 0) return;
+    __threadfence();
+    const unsigned long long kk = (unsigned long long)p.k;
+    const unsigned long long R = __ldcg(c.outc), Wn = __ldcg(c.bufc);
+    if ((__ldcg(&st->error) & 2u) == 0 && R < kk && kk <= R + Wn) {
+      st->K = kk - R;  // a fresh select of K - R among the Wn window members (pass 0 runs on them)
+      st->C = Wn;
+      st->Cp = Wn;
+      st->src1 = sslot + 1;
+      st->buf_count[sslot == 1 ? 0 : 1] = 0;
+    } else {
+      st->win_state = 2;  // miss: pass 0 re-reads L and the paper's passes follow
+      st->out_count = 0;
+      st->buf_count[sslot] = 0;
+      st->error &= ~2u;
+    }
+    st->ticket = 0;
+    return;
+  }
 
   if (!hist_on) return;
 
@@ -155,31 +197,172 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pass_kernel(const GridPara
   __threadfence();
 
   const unsigned long long kk = (unsigned long long)p.k;
-  const unsigned long long Kin = (DF == 0) ? kk : st->K;
-  const unsigned long long Cin = Cprev;  // elements counted by this histogram
+  unsigned long long Kin = (FILTER || redo_buf) ? st->K : kk;
+  unsigned long long Cin = Cprev;  // elements counted by this histogram
   const ScanResult r = scan_choose<kBlock>(
       [&](int b) { return (unsigned long long)__ldcg(&gh[b]); }, nb, Kin, sh_tmp, &sh_res);
   CountT* gh2 = (CountT*)p.ghist + ((size_t)row * 2 + ((q + 1) & 1)) * kMaxBins;
   for (int i = tid; i < kMaxBins; i += kBlock) gh2[i] = 0;
   if (tid == 0) {
-    const unsigned long long newK = Kin - r.before, newC = r.cnt;   // Alg1 L26-28
-    st->Cp = Cin;
-    st->C = newC;
-    st->K = newK;
-    if (!dh.is_idx) st->tcode |= (unsigned long long)r.j << dh.shift;
-    else st->tidx |= (unsigned long long)r.j << dh.shift;
-    st->j = r.j;
-    st->npass = q + 1;
-    if (newK == newC) st->stop1 = q + 1;                             // early stop
-    st->buf_count[(q + 1) & 1] = 0;
+    int next_src1 = (c.store) ? sslot + 1 : src1;  // the buffer this pass wrote feeds the next one
+    {
+      const unsigned long long newK = Kin - r.before, newC = r.cnt;   // Alg1 L26-28
+      st->Cp = Cin;
+      st->C = newC;
+      st->K = newK;
+      if (!dh.is_idx) st->tcode |= (unsigned long long)r.j << dh.shift;
+      else st->tidx |= (unsigned long long)r.j << dh.shift;
+      st->j = r.j;
+      st->npass = q + 1;
+      if (newK == newC) st->stop1 = q + 1;                             // early stop
+      st->src1 = next_src1;
+      st->buf_count[next_src1 == 1 ? 1 : 0] = 0;                        // next pass's output buffer
+      if (r.total != Cin) st->error |= 4u;
+      if (p.trace && q < kTraceMaxPasses) {
+        int64_t* t = p.trace + ((size_t)row * kTraceMaxPasses + q) * kTraceFields;
+        t[0] = dh.width; t[1] = c.srcL; t[2] = c.store; t[3] = r.j; t[4] = (int64_t)newK; t[5] = (int64_t)newC;
+        t[6] = (int64_t)Cin; t[7] = (int64_t)__ldcg(c.outc); t[8] = (newK == newC); t[9] = (int64_t)nread;
+      }
+    }
     st->ticket = 0;
-    if (r.total != Cin) st->error |= 4u;
-    if (p.trace && q < kTraceMaxPasses) {
-      int64_t* t = p.trace + ((size_t)row * kTraceMaxPasses + q) * kTraceFields;
-      t[0] = dh.width; t[1] = c.srcL; t[2] = c.store; t[3] = r.j; t[4] = (int64_t)newK; t[5] = (int64_t)newC;
-      t[6] = (int64_t)Cin; t[7] = (int64_t)__ldcg(c.outc); t[8] = (newK == newC); t[9] = (int64_t)nread;
+  }
+}
+
+// Sample-guided window: one CTA per row reads S
+// stratified samples, selects the sample order statistics at ranks r -/+ margin around the expected
+// rank of the K-th key, and stores them as the window [lo, hi]. Exactness never depends on it: the
+// window pass validates the window and falls back to the paper's passes when it misses.
+constexpr int kSampleBlock = 1024;
+constexpr int kMaxSamples = 16384;
+
+template <typename W>
+__device__ W block_select_rank(const W* a, int n, int rank, int bits, unsigned* hist, W* shw) {
+  // MSD radix select (8-bit digits) of the element of rank `rank` (0-based) among a[0..n) in shared
+  // memory; the 256-bin scan is done by warp 0 (8 bins per lane + shuffle scan).
+  W prefix = 0, pmask = 0;
+  int rk = rank;
+  const int lane = threadIdx.x & 31;
+  for (int hi = bits; hi > 0; hi -= 8) {
+    const int w = hi < 8 ? hi : 8, sh = hi - w;
+    for (int i = threadIdx.x; i < 256; i += blockDim.x) hist[i] = 0;
+    __syncthreads();
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+      const W v = a[i];
+      if ((v & pmask) == prefix) atomicAdd(&hist[(unsigned)(v >> sh) & 255u], 1u);
+    }
+    __syncthreads();
+    if (threadIdx.x < 32) {
+      unsigned c[8], tot = 0;
+#pragma unroll
+      for (int t = 0; t < 8; ++t) { c[t] = hist[lane * 8 + t]; tot += c[t]; }
+      unsigned incl = tot;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+      }
+      unsigned run = incl - tot;  // bins before this lane's 8
+      if (run <= (unsigned)rk && (unsigned)rk < incl) {
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+          if (run <= (unsigned)rk && (unsigned)rk < run + c[t]) {
+            shw[0] = (W)(lane * 8 + t);
+            shw[1] = (W)run;
+          }
+          run += c[t];
+        }
+      }
+    }
+    __syncthreads();
+    const W d = shw[0];
+    rk -= (int)shw[1];
+    prefix |= d << sh;
+    pmask |= (W)((1u << w) - 1u) << sh;
+    __syncthreads();
+  }
+  return prefix;
+}
+
+constexpr int kSampleCTAs = 16;  // CTAs per row issuing the scattered sample loads (one SM cannot
+                                 // keep 16K independent DRAM loads in flight)
+
+template <int KIND>
+__global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p, int nsamp) {
+  using U = typename KT<KIND>::U;
+  using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
+  extern __shared__ __align__(16) unsigned char sample_smem[];
+  W* codes = (W*)sample_smem;  // nsamp codes (last CTA only)
+  __shared__ unsigned hist[256];
+  __shared__ W shw[2];
+  __shared__ int sh_last;
+  const int64_t row = blockIdx.x / kSampleCTAs;
+  const int part = blockIdx.x % kSampleCTAs;
+  RowState* st = p.st + row;
+  pdl_wait();
+  pdl_trigger();
+  const U* rowp = (const U*)p.keys + row * p.len;
+  W* samp = (W*)p.samp + row * (int64_t)nsamp;
+  const U xmask = p.sel_min ? (U)0 : (U)~(U)0;
+  const int64_t stride = p.len / nsamp;
+  // phase 1: stratified samples s = part, part + 16, ... (all of this CTA's loads in flight at once)
+  {
+    constexpr int PER = kMaxSamples / (kSampleBlock * kSampleCTAs);
+    W v[PER];
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+      const int s = (t * kSampleBlock + threadIdx.x) * kSampleCTAs + part;
+      v[t] = (s < nsamp) ? (W)to_code_x<KIND>(__ldg(rowp + (int64_t)s * stride + stride / 2), xmask) : (W)0;
+    }
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+      const int s = (t * kSampleBlock + threadIdx.x) * kSampleCTAs + part;
+      if (s < nsamp) samp[s] = v[t];
     }
   }
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) sh_last = (atomicAdd(&st->ticket, 1u) == (unsigned)(kSampleCTAs - 1));
+  __syncthreads();
+  if (!sh_last) return;
+  __threadfence();
+  // phase 2 (last CTA of the row): the window from the sample order statistics
+  for (int s = threadIdx.x; s < nsamp; s += blockDim.x) codes[s] = __ldcg(samp + s);
+  __syncthreads();
+  if (threadIdx.x == 0) st->ticket = 0;
+  // expected sample rank of the K-th key and a 3.5-sigma (+3) margin of the binomial sample count:
+  // a miss (probability < 1e-3) only costs the fallback, never exactness
+  const double f = (double)p.k / (double)p.len;
+  const double r = f * nsamp;
+  const double m = 3.5 * sqrt(r * (1.0 - f)) + 3.0;
+  const int rlo = (int)floor(r - m), rhi = (int)ceil(r + m);
+  if (rhi >= nsamp - 1) {  // the window would hold most of the row: keep the paper's passes
+    if (threadIdx.x == 0) st->win_state = 0;
+    return;
+  }
+  const W lo = (rlo <= 0) ? (W)0 : block_select_rank<W>(codes, nsamp, rlo, KT<KIND>::R, hist, shw);
+  const W hi = block_select_rank<W>(codes, nsamp, rhi, KT<KIND>::R, hist, shw);
+  if (threadIdx.x == 0) {
+    st->win_lo = lo;
+    st->win_hi = hi;
+    st->win_state = 1;
+  }
+}
+
+// Launch with programmatic stream serialisation (PDL): the kernel may start while the previous one
+// drains; it synchronises with pdl_wait() before touching anything the previous kernel wrote.
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, args...);
 }
 
 struct Events {
@@ -196,34 +379,49 @@ constexpr size_t hist_smem_bytes() {
 }
 
 template <int KIND, typename IdxT, int DF, int DH, bool HASIDX>
-cudaError_t launch_one(const GridParams& gp, unsigned grid, int q, cudaStream_t s) {
+cudaError_t launch_one(const GridParams& gp, unsigned grid, int q, int redo, cudaStream_t s) {
   constexpr size_t smem = hist_smem_bytes<KIND, IdxT, DF, DH>();
   static const cudaError_t attr = cudaFuncSetAttribute(pass_kernel<KIND, IdxT, DF, DH, HASIDX>,
                                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (attr != cudaSuccess) return attr;
-  pass_kernel<KIND, IdxT, DF, DH, HASIDX><<<grid, kBlock, smem, s>>>(gp, q);
-  return cudaSuccess;
+  return launch_pdl(pass_kernel<KIND, IdxT, DF, DH, HASIDX>, dim3(grid), dim3(kBlock), smem, s, gp, q, redo);
 }
 
 template <int KIND, typename IdxT, bool HASIDX>
-cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, const Events& ev, cudaStream_t s) {
+cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, const Events& ev, cudaStream_t s) {
   const unsigned grid = (unsigned)((long long)batch * gp.cpr);
-  ev.record(0, s);
+  int ie = 0;
+  ev.record(ie++, s);
+  if (nsamp > 0) {  // sample-guided window: sample, window pass (= pass 0 + filter), pass 0 over the window
+    using W = std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long, unsigned>;
+    const size_t smem = (size_t)kMaxSamples * sizeof(W);
+    static const cudaError_t attr =
+        cudaFuncSetAttribute(sample_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (attr != cudaSuccess) return attr;
+    cudaError_t es = launch_pdl(sample_kernel<KIND>, dim3((unsigned)(batch * kSampleCTAs)), dim3(kSampleBlock),
+                                (size_t)nsamp * sizeof(W), s, gp, nsamp);
+    if (es != cudaSuccess) return es;
+    ev.record(ie++, s);
+    cudaError_t e = launch_one<KIND, IdxT, 3, 0, HASIDX>(gp, grid, 0, 0, s);
+    if (e != cudaSuccess) return e;
+    ev.record(ie++, s);
+  }
   for (int q = 0; q <= gp.P; ++q) {
     const int DF = q == 0 ? 0 : (digit_of(q - 1, KT<KIND>::R, gp.IB).is_idx ? 2 : 1);
     const int DH = q == gp.P ? 0 : (digit_of(q, KT<KIND>::R, gp.IB).is_idx ? 2 : 1);
     const int v = DF * 3 + DH;
     cudaError_t e;
+    const int redo = (q == 0 && nsamp > 0) ? 1 : 0;
     switch (v) {
-      case 0 * 3 + 1: e = launch_one<KIND, IdxT, 0, 1, HASIDX>(gp, grid, q, s); break;
-      case 1 * 3 + 1: e = launch_one<KIND, IdxT, 1, 1, HASIDX>(gp, grid, q, s); break;
-      case 1 * 3 + 2: e = launch_one<KIND, IdxT, 1, 2, HASIDX>(gp, grid, q, s); break;
-      case 2 * 3 + 2: e = launch_one<KIND, IdxT, 2, 2, HASIDX>(gp, grid, q, s); break;
-      case 2 * 3 + 0: e = launch_one<KIND, IdxT, 2, 0, HASIDX>(gp, grid, q, s); break;
+      case 0 * 3 + 1: e = launch_one<KIND, IdxT, 0, 1, HASIDX>(gp, grid, q, redo, s); break;
+      case 1 * 3 + 1: e = launch_one<KIND, IdxT, 1, 1, HASIDX>(gp, grid, q, 0, s); break;
+      case 1 * 3 + 2: e = launch_one<KIND, IdxT, 1, 2, HASIDX>(gp, grid, q, 0, s); break;
+      case 2 * 3 + 2: e = launch_one<KIND, IdxT, 2, 2, HASIDX>(gp, grid, q, 0, s); break;
+      case 2 * 3 + 0: e = launch_one<KIND, IdxT, 2, 0, HASIDX>(gp, grid, q, 0, s); break;
       default: return cudaErrorInvalidValue;
     }
     if (e != cudaSuccess) return e;
-    ev.record(q + 1, s);
+    ev.record(ie++, s);
   }
   return cudaGetLastError();
 }
@@ -231,9 +429,9 @@ cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, const Events
 template <int KIND>
 cudaError_t launch_grid_kind(const SelectArgs& a, const Plan& pl, const GridParams& gp, cudaStream_t s) {
   const Events ev{a.events, a.n_events};
-  if (a.in_idx) return launch_grid_passes<KIND, uint64_t, true>(gp, a.batch, ev, s);
-  if (pl.idx64) return launch_grid_passes<KIND, uint64_t, false>(gp, a.batch, ev, s);
-  return launch_grid_passes<KIND, uint32_t, false>(gp, a.batch, ev, s);
+  if (a.in_idx) return launch_grid_passes<KIND, uint64_t, true>(gp, a.batch, 0, ev, s);
+  if (pl.idx64) return launch_grid_passes<KIND, uint64_t, false>(gp, a.batch, pl.nsamp, ev, s);
+  return launch_grid_passes<KIND, uint32_t, false>(gp, a.batch, pl.nsamp, ev, s);
 }
 
 #define AIRTOPK_INSTANTIATE_GRID(KIND) \

@@ -22,6 +22,9 @@
 
 namespace airtopk {
 
+#ifndef AIRTOPK_SLOW_REG
+#define AIRTOPK_SLOW_REG 0
+#endif
 constexpr int kUnroll = 4;
 constexpr int kQCap = 64;
 // Copies of the shared histogram in the filter passes: lane l counts into copy l % kHistCopies
@@ -48,7 +51,7 @@ struct WarpQ {
 template <int KIND, typename IdxT, int DF>
 __host__ __device__ constexpr int hist_copies() {
   using U = typename KT<KIND>::U;
-  return (DF == 0) ? 1 : (sizeof(U) + sizeof(IdxT) <= 8 ? kHistCopies : 2);
+  return (DF == 0 || DF == 3) ? 1 : (sizeof(U) + sizeof(IdxT) <= 8 ? kHistCopies : 2);
 }
 
 // Flush a warp queue: ONE global atomic reserves n slots, then coalesced stores. Out of line so the
@@ -100,6 +103,20 @@ __device__ __forceinline__ void wq_push(WarpQ<typename KT<KIND>::U, IdxT>* wq, i
   cnt += n;
 }
 
+// Element b (0 .. kUnroll*VEC-1) of a thread's tile registers, selected without local memory.
+template <typename U>
+__device__ __forceinline__ U tile_elem(const uint4 (&r)[kUnroll], int b) {
+  constexpr int VEC = 16 / sizeof(U);
+  const int u = b / VEC, e = b % VEC;
+  uint4 v = r[0];
+#pragma unroll
+  for (int i = 1; i < kUnroll; ++i) v = (u == i) ? r[i] : v;
+  U out = vec_elem<U>(v, 0);
+#pragma unroll
+  for (int i = 1; i < VEC; ++i) out = (e == i) ? vec_elem<U>(v, i) : out;
+  return out;
+}
+
 // Everything one pass of one row needs (built by the engine from its copy of the row state).
 template <typename U, typename IdxT>
 struct PassCtx {
@@ -126,6 +143,7 @@ struct PassCtx {
   unsigned long long* bufc;
   unsigned long long capa;
   unsigned* err;
+  unsigned long long lo, span1;  // DF == 3 window: candidates lo <= code < lo + span1, results code < lo
   unsigned* hist;  // shared, kMaxBins * hist_copies() counters, zeroed by the caller
   WarpQ<U, IdxT>* oq;
   WarpQ<U, IdxT>* bq;
@@ -179,9 +197,14 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
     wq_push<KIND, IdxT>(c.bq, bcnt, pred, code, idx, c.bufc, c.capa, c.bco, c.bio, 1, sel_min, c.err);
   };
   // Filter classification of digit q-1 (Alg1 L15-22): win = result, cand = candidate for pass q.
+  const W wlo = (W)c.lo, wspan = (W)c.span1;
   auto classify = [&](U code, IdxT idx, bool valid, bool& win, bool& cand) {
     bool lt, eq;
-    if constexpr (DF == 1) {
+    if constexpr (DF == 3) {  // sample-guided window
+      win = valid && ((W)code < wlo);
+      cand = valid && ((W)((W)code - wlo) < wspan);
+      return;
+    } else if constexpr (DF == 1) {
       const W h = (W)code >> sf;
       lt = (W)(h - bc) < (W)(tc - bc);
       eq = (h == tc);
@@ -242,7 +265,20 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
         return;
       }
       unsigned fl = 0;  // elements that must leave through the queues (results / stored candidates)
-      if constexpr (DF == 1 && DH == 1) {
+      if constexpr (DF == 3) {
+        // window pass: results below the window -> output, window members -> candidate buffer;
+        // pure filter (no histogram): a miss is repaired by re-running the paper's pass 1
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+          const bool valid = FULL || (vb + (int64_t)u * BLOCK < vlim);
+#pragma unroll
+          for (int e = 0; e < VEC; ++e) {
+            const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
+            const bool sel = ((W)code < wlo) || ((W)((W)code - wlo) < wspan);
+            if (valid && sel) fl |= 1u << (u * VEC + e);
+          }
+        }
+      } else if constexpr (DF == 1 && DH == 1) {
         // adjacent key digits: y = (code >> shh) - B places the elements whose higher digits match
         // the prefix at [S, S + nb) and the results below S (see the derivation at kx_* below)
 #pragma unroll
@@ -290,7 +326,11 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
         const int b = has ? __ffs(fl) - 1 : 0;
         fl &= fl - 1;
         const int64_t pos = head + (vb + (int64_t)(b / VEC) * BLOCK) * VEC + (b % VEC);
+#if AIRTOPK_SLOW_REG
+        const U code = to_code_x<KIND>(tile_elem<U>(r, b), xmask);
+#else
         const U code = to_code_x<KIND>(has ? __ldcg(rowp + pos) : (U)0, xmask);
+#endif
         const IdxT idx = has ? index_of(pos) : (IdxT)0;
         bool w, cd;
         classify(code, idx, has, w, cd);
@@ -328,7 +368,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
         const IdxT idx = valid ? index_of(i) : (IdxT)0;
         bool win, cand;
         classify(code, idx, valid, win, cand);
-        hist_cand(code, idx, cand);
+        if constexpr (DF != 3) hist_cand(code, idx, cand);
         push_out(win, code, idx);
         if (store) push_buf(cand, code, idx);
       }
@@ -344,7 +384,14 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
     const unsigned long long e0 = std::min<unsigned long long>(n, (unsigned long long)c.slice * per);
     const unsigned long long e1 = std::min<unsigned long long>(n, e0 + per);
     nread = n;
-    if constexpr (DF != 0) {
+    if constexpr (DF == 0) {
+      for (unsigned long long base = e0; base < e1; base += BLOCK) {
+        const unsigned long long i = base + tid;
+        const bool valid = i < e1;
+        const U code = valid ? c.bcin[i] : (U)0;
+        shared_inc(hbase + 4u * (valid ? (unsigned)(((W)code >> shh) & hmask) : (unsigned)kDummyBin));
+      }
+    } else if constexpr (DF != 3) {
       for (unsigned long long base = e0; base < e1; base += BLOCK) {
         const unsigned long long i = base + tid;
         const bool valid = i < e1;

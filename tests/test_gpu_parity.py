@@ -169,7 +169,7 @@ def test_trace_matches_algorithm1(dist, m, k, alpha):
     x = gen.keys(dist, 55, n, m_bits=m)
     tr = at.trace_buffer(1)
     xd = to_device(x, "f32").reshape(1, -1)
-    at.select(xd, k, alpha=alpha, trace=tr, engine=at.ENGINE_GRID)
+    at.select(xd, k, alpha=alpha, trace=tr, engine=at.ENGINE_GRID, window=-1)  # the paper's passes
     torch.cuda.synchronize()
     g = tr.cpu().numpy()[0]
     codes = oracle.codes(x)
@@ -263,3 +263,52 @@ def test_cluster_engine_alpha(alpha):
     x = _keys("adversarial", 13, 6, 1 << 17, 10)
     v, i = gpu_select(x, "f32", 3000, alpha=alpha, engine=2)
     assert_parity(x, "f32", 3000, True, v, i)
+
+
+# ---------------------------------------------------------------- sample-guided window (NEXT #1)
+
+def _sample_positions(n):
+    ns = min(max(n // 256, 1024), 16384, n)
+    stride = n // ns
+    return np.arange(ns, dtype=np.int64) * stride + stride // 2
+
+
+@pytest.mark.parametrize("window", [-1, 1])
+@pytest.mark.parametrize("dist,m", [("uniform", 20), ("normal", 20), ("adversarial", 20), ("adversarial", 12)])
+@pytest.mark.parametrize("k", [1, 100, 77777, 1 << 19])
+def test_window_on_off(window, dist, m, k):
+    x = _keys(dist, 71, 2, 1 << 20, m)
+    for sm in (True, False):
+        v, i = gpu_select(x, "f32", k, sm, window=window, engine=1)
+        assert_parity(x, "f32", k, sm, v, i)
+
+
+@pytest.mark.parametrize("case", ["high", "low", "ties"])
+def test_window_fallback(case):
+    """Inputs built so the stratified sample misrepresents the row: the window pass must detect the
+    miss (R >= K or K > R + W) and fall back to the paper's passes, exactly."""
+    n = 1 << 20
+    x = gen.uniform_f32(8, n)
+    pos = _sample_positions(n)
+    if case == "high":
+        x[pos] = np.float32(1e30)
+        ks = (1000, 500000)
+    elif case == "low":
+        x[pos] = np.float32(-1e30)
+        ks = (len(pos) + 5, 500000)
+    else:
+        x[:] = np.float32(3.0)
+        x[pos] = np.float32(2.0)
+        ks = (1, len(pos) + 1, 700000)
+    for k in ks:
+        v, i = gpu_select(x, "f32", k, True, window=1, engine=1)
+        assert_parity(x, "f32", k, True, v, i)
+
+
+def test_window_describe():
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    d = at.describe(torch.float32, 1, 1 << 30, 1 << 20)
+    assert d["engine"] == 1 and d["launches"] == d["passes"] + 3
+    d = at.describe(torch.float32, 1, 1 << 30, 1 << 20, window=-1)
+    assert d["launches"] == d["passes"] + 1
