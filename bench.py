@@ -176,6 +176,11 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=10.0)
     ap.add_argument("--ref-budget", type=float, default=20.0)
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--engine", type=int, default=0, help="0 auto, 1 grid, 2 cluster (ablations)")
+    ap.add_argument("--window", type=int, default=0, help="sample-guided window: 0 auto, 1 on, -1 off (ablation)")
+    ap.add_argument("--tma", type=int, default=0, help="bulk-copy streaming: 0 auto, 1 on, -1 off (ablation)")
+    ap.add_argument("--dist-backend", default="nccl", help="nccl (default); gloo only to self-test the "
+                    "multi-rank flow with several ranks on one GPU")
     args = ap.parse_args()
     if args.steps is None:
         args.steps = DEFAULT_STEPS[args.config]
@@ -193,11 +198,16 @@ def main():
     import paper_conf_sc_zhangnlw23_b200 as at
     from paper_conf_sc_zhangnlw23_b200 import dist as atdist
 
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    ndev = torch.cuda.device_count()
+    local_dev = local % max(1, ndev)  # (> 1 rank per GPU only for the --dist-backend gloo self-test)
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        dist.init_process_group("nccl", device_id=dev)
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(args.dist_backend)
     at.lib()
 
     cfg = args.config
@@ -220,16 +230,18 @@ def main():
         split = world > 1
     k = c["k"]
     xd = torch.from_numpy(xh).to(dev)
-    ws = torch.empty(max(1, at.workspace_bytes(torch.float32, batch, n, k)), dtype=torch.uint8, device=dev)
+    sel_opts = dict(engine=args.engine, window=args.window, tma=args.tma)
+    ws = torch.empty(max(1, at.describe(torch.float32, batch, n, k, **sel_opts)["workspace_bytes"]),
+                     dtype=torch.uint8, device=dev)
     ov = torch.empty((batch, k), dtype=torch.float32, device=dev)
     oi = torch.empty((batch, k), dtype=torch.int64, device=dev)
-    plan = at.describe(torch.float32, batch, n, k)
+    plan = at.describe(torch.float32, batch, n, k, **sel_opts)
     n_launch = plan["launches"]
     stream = torch.cuda.current_stream(dev)
     ev_sets = []
 
     def step(events=None):
-        v, i = at.select(xd, k, workspace=ws, out=(ov, oi), events=events)
+        v, i = at.select(xd, k, workspace=ws, out=(ov, oi), events=events, **sel_opts)
         if split:
             gv, gi = atdist.select_split_row(xd.reshape(-1), k, total_len=world * n, shard_offset=rank * n,
                                              select_fn=lambda t, kk, lg: (v.reshape(-1), i.reshape(-1)))
@@ -288,7 +300,8 @@ def main():
     out_bytes = batch * k * (4 + 8)
     # algorithmic bytes of the dominant kernel: passes that read the input read N*4 bytes once
     # (grid engine: launch 0 and 1 read L; cluster engine: its single launch reads the rows)
-    dom_alg = in_bytes if dom <= 1 else None
+    names, reads_L = launch_names(plan)
+    dom_alg = in_bytes if reads_L[dom] else None
     value = total_units / (ms * 1e-3)
 
     # ---------------- correctness spot check of the timed configuration (sampled, no oracle):
@@ -300,10 +313,9 @@ def main():
         roofline = None
         if dom_alg is not None:
             ach = dom_alg / (per[dom] * 1e-3) / 1e9
-            kname = f"pass_kernel q={dom}" if plan["engine"] == 1 else "cluster_kernel"
-            roofline = {"bound": "hbm", "kernel": kname, "achieved": ach, "peak": peak,
+            roofline = {"bound": "hbm", "kernel": names[dom], "achieved": ach, "peak": peak,
                         "peak_kind": peak_kind, "unit": "GB/s", "frac": ach / peak,
-                        "traffic": load_traffic(cfg, dom),
+                        "traffic": load_traffic(cfg, dom, n_launch),
                         "alg_bytes_per_launch": dom_alg, "launch_ms": float(per[dom])}
         whole = (in_bytes + out_bytes) / (select_ms * 1e-3) / 1e9
         result = {
@@ -364,19 +376,42 @@ def main():
         dist.destroy_process_group()
 
 
+def launch_names(plan):
+    """Names of a select's launches in order, and whether each streams the input row L once (its
+    algorithmic bytes are then N*4; SURVEY §8(d) per-element figure x elements per launch)."""
+    if plan["engine"] == 2:
+        return ["cluster_kernel (all passes)"], [True]
+    if plan["engine"] == 3:
+        return ["trivial_copy"], [True]
+    P = plan["passes"]
+    window = plan["launches"] == P + 3
+    names, reads = [], []
+    if window:
+        names += ["sample_kernel", "window_pass (DF=3)"]
+        reads += [False, True]
+    for q in range(P + 1):
+        nm = "last_filter (q=P)" if q == P else f"pass_kernel q={q}"
+        names.append(nm + (" [window buffer]" if window and q <= 1 else ""))
+        reads.append((not window) and q <= 1)
+    return names, reads
+
+
 def plan_merge_launches(world, k):
     import torch
     import paper_conf_sc_zhangnlw23_b200 as at
     return at.describe(torch.float32, 1, world * k, k)["launches"]
 
 
-def load_traffic(cfg, q):
-    """dram bytes (read+write) per launch of kernel q from the committed ncu summary, if any."""
-    p = os.path.join(ROOT, "profiles", "traffic.json")
+def load_traffic(cfg, q, n_launch):
+    """dram bytes (read + write) of launch q of a select, from the committed ncu launch list
+    (profiles/traffic_launches.json, written by tools/make_profiles.py from `ncu --metrics
+    dram__bytes_read.sum,dram__bytes_write.sum`): the second select of the list (warm), else the first."""
+    p = os.path.join(ROOT, "profiles", "traffic_launches.json")
     try:
         with open(p) as f:
-            d = json.load(f)
-        return d.get(cfg, {}).get(str(q))
+            d = json.load(f).get(cfg, {})
+        v = d.get(str(n_launch + q), d.get(str(q)))
+        return float(v) if v is not None else None
     except Exception:
         return None
 

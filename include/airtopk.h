@@ -100,7 +100,8 @@ typedef struct {
                            events on the launching stream. NULL = none. */
   int32_t window;       /* sample-guided window pass: 0 = auto (grid engine,
                            len >= 2^18), 1 = on, -1 = off (the paper's passes only). Exact either way. */
-  int32_t reserved1;
+  int32_t tma;          /* grid engine streaming: 0 = auto (bulk-copy rings for a few long rows), 1 = bulk
+                           copies (cp.async.bulk + mbarrier per-warp rings), -1 = register loads. */
 } airtopk_options;
 
 #define AIRTOPK_TRACE_MAX_PASSES 16
@@ -147,8 +148,9 @@ airtopk_status airtopk_select_with_idx(const void* keys, const int64_t* in_idx, 
 
 /* End-to-end convenience with HOST buffers: copies keys host->device, selects, copies the results
  * device->host and SYNCHRONISES `stream` before returning. Pinned (page-locked) host memory gives
- * asynchronous DMA; pageable memory works but is staged by the driver. Device scratch comes from
- * cudaMallocAsync on `stream`. */
+ * asynchronous DMA; pageable memory works but is staged by the driver. Device staging (keys,
+ * outputs, workspace) is a per-thread, per-device cudaMalloc cache that grows on demand and is
+ * released when the calling thread exits. */
 airtopk_status airtopk_select_host(const void* h_keys, airtopk_dtype dtype, int64_t batch, int64_t len,
                                    int64_t k, int select_min, void* h_out_vals, int64_t* h_out_idx,
                                    airtopk_stream_t stream);

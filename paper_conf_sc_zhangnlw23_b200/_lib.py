@@ -36,7 +36,7 @@ class Options(ctypes.Structure):
         ("trace", ctypes.c_void_p),
         ("events", ctypes.c_void_p),
         ("window", ctypes.c_int32),
-        ("reserved1", ctypes.c_int32),
+        ("tma", ctypes.c_int32),
     ]
 
 

@@ -5,6 +5,7 @@
 // stream (the iteration-fused property: the CPU only launches kernels, P:50/P:142/P:158).
 #include <algorithm>
 #include <cstdlib>
+#include <cmath>
 #include <cstring>
 
 #include "../../include/airtopk.h"
@@ -75,11 +76,14 @@ Plan make_plan(const SelectArgs& a) {
   p.off_hist = align_up(sizeof(RowState) * (size_t)a.batch, 256);
   p.off_bcode = p.off_hist + align_up((size_t)a.batch * 2 * kMaxBins * csz, 256);
   p.off_bidx = p.off_bcode + align_up((size_t)2 * a.batch * p.cap_alloc * key_bytes(a.kind), 256);
-  // sample-guided window (grid engine, position indices): ~len/256 stratified samples, 1K..16K
+  // sample-guided window (grid engine, position indices): stratified samples, 4K..16K
   p.nsamp = 0;
   if (!a.in_idx && (a.window > 0 || (a.window == 0 && a.len >= (int64_t(1) << 18)))) {
-    int64_t ns = std::min<int64_t>(std::max<int64_t>(a.len / 256, 1024), 16384);
-    p.nsamp = (int)std::min<int64_t>(ns, a.len);
+    // samples are read in whole 128-byte lines (32 consecutive elements): len/64 capped at 16K
+    // costs <= 1/64 of the row's bytes; at least 4K samples keep the window small vs N/alpha
+    int64_t ns = std::min<int64_t>(std::max<int64_t>(a.len / 128, 4096), 16384);
+    ns = std::min<int64_t>(ns, a.len / 2) / 32 * 32;
+    p.nsamp = ns >= 1024 ? (int)ns : 0;
   }
   p.off_samp = p.off_bidx + align_up((size_t)2 * a.batch * p.cap_alloc * isz, 256);
   p.bytes = p.off_samp + align_up((size_t)a.batch * p.nsamp * (key_bytes(a.kind) == 8 ? 8 : 4), 256);
@@ -89,6 +93,7 @@ Plan make_plan(const SelectArgs& a) {
 // Engine choice: the cluster engine (one launch, DSMEM scans) for batched
 // and small rows, the grid engine (one launch per pass, whole GPU per row) for long rows.
 static int auto_engine(const SelectArgs& a) {
+  if (a.window > 0 && !a.in_idx) return 1;  // window requested: grid window pass (+ cluster tail)
   if (a.len <= (int64_t(1) << 17)) return 2;
   if (a.len <= (int64_t(1) << 22) && a.batch >= 16 && getenv("AIRTOPK_CLUSTER_BATCHED")) return 2;
   return 1;
@@ -109,11 +114,29 @@ static void choose_launch(const SelectArgs& a, Plan& p) {
     p.csize = auto_cluster_size(a);
     return;
   }
+  // expected window size per row (entries) -> tail mode for small windows
+  p.tail = 0;
+  if (p.nsamp > 0 && a.window >= 0) {
+    const double f = (double)a.k / (double)a.len, r = f * p.nsamp;
+    const double rhi = r + 4.0 * std::sqrt(r * (1.0 - f)) + 9.0;  // sample_kernel's margin
+    const double expect = rhi / p.nsamp * (double)a.len;
+    if (expect <= (double)(1 << 20) && a.engine == 0) {
+      p.tail = 1;
+      int cs = 1;
+      while (cs < 16 && cs * 16384.0 < expect) cs <<= 1;
+      p.csize = a.cluster_size > 0 ? a.cluster_size : cs;
+    }
+  }
+  // bulk-copy streaming for a few long rows (every SM busy with 1 CTA); register loads otherwise
+  p.tma = 0;
+  if (!a.in_idx && !p.idx64 && a.tma >= 0 &&
+      (a.tma > 0 || (a.batch * 2 <= num_sms() && a.len >= (int64_t(1) << 22))))
+    p.tma = 1;
   if (a.ctas_per_row > 0) {
     p.cpr = a.ctas_per_row;
     return;
   }
-  const int64_t target = (int64_t)num_sms() * grid_blocks_per_sm(a, p.idx64);
+  const int64_t target = (int64_t)num_sms() * (p.tma ? 1 : grid_blocks_per_sm(a, p.idx64));
   const int64_t chunk = grid_vec_chunk(a.kind);
   const int64_t maxc = std::max<int64_t>(1, (a.len + chunk - 1) / chunk);
   // whole waves: batch x cpr <= target CTAs (a partial second wave costs more than idle slots)
@@ -175,6 +198,7 @@ static SelectArgs make_args(const void* keys, int dt, int64_t batch, int64_t len
     a.events = opt->events;
     a.n_events = opt->events ? opt->n_events : 0;
     a.window = opt->window;
+    a.tma = opt->tma;
   }
   if (a.alpha == 0) a.alpha = 128;
   return a;
@@ -275,9 +299,32 @@ airtopk_status airtopk_select_host(const void* h_keys, airtopk_dtype dtype, int6
   Plan p = make_plan(a);
   const size_t ws_b = p.engine == 3 ? 0 : p.bytes;
   const size_t o1 = align_up(in_b, 256), o2 = o1 + align_up(ov_b, 256), o3 = o2 + align_up(oi_b, 256);
-  char* d = nullptr;
-  cudaError_t e = cudaMallocAsync((void**)&d, o3 + ws_b, s);
+  // device staging cached per thread and device (this call synchronises before returning, so the
+  // next call on this thread may reuse it); grows on demand, released at thread exit
+  struct Staging {
+    char* ptr = nullptr;
+    size_t bytes = 0;
+    int dev = -1;
+    ~Staging() { if (ptr) cudaFree(ptr); }
+  };
+  static thread_local Staging stg;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return fail_cuda(e);
+  if (stg.dev != dev || stg.bytes < o3 + ws_b) {
+    if (stg.ptr) {
+      cudaStreamSynchronize(s);
+      cudaFree(stg.ptr);
+      stg.ptr = nullptr;
+    }
+    if ((e = cudaMalloc((void**)&stg.ptr, o3 + ws_b)) != cudaSuccess) {
+      stg.bytes = 0;
+      return fail_cuda(e);
+    }
+    stg.bytes = o3 + ws_b;
+    stg.dev = dev;
+  }
+  char* d = stg.ptr;
   airtopk_status st = AIRTOPK_OK;
   if ((e = cudaMemcpyAsync(d, h_keys, in_b, cudaMemcpyHostToDevice, s)) != cudaSuccess) st = fail_cuda(e);
   if (st == AIRTOPK_OK) {
@@ -290,7 +337,6 @@ airtopk_status airtopk_select_host(const void* h_keys, airtopk_dtype dtype, int6
     st = fail_cuda(e);
   if (st == AIRTOPK_OK && (e = cudaMemcpyAsync(h_out_idx, d + o2, oi_b, cudaMemcpyDeviceToHost, s)) != cudaSuccess)
     st = fail_cuda(e);
-  cudaFreeAsync(d, s);
   if ((e = cudaStreamSynchronize(s)) != cudaSuccess && st == AIRTOPK_OK) st = fail_cuda(e);
   return st;
 }
@@ -308,9 +354,9 @@ airtopk_status airtopk_describe(airtopk_dtype dtype, int64_t batch, int64_t len,
   std::memset(out, 0, sizeof(*out));
   out->engine = p.engine;
   out->passes = p.P;
-  out->launches = p.engine == 3 ? 1 : (p.engine == 2 ? 1 : p.P + 1 + (p.nsamp > 0 ? 2 : 0));
+  out->launches = p.engine == 3 ? 1 : (p.engine == 2 ? 1 : (p.tail ? 3 : p.P + 1 + (p.nsamp > 0 ? 2 : 0)));
   out->ctas_per_row = p.engine == 1 ? p.cpr : 0;
-  out->cluster_size = p.engine == 2 ? p.csize : 0;
+  out->cluster_size = (p.engine == 2 || p.tail) ? p.csize : 0;
   out->index_bits = p.IB;
   out->buffer_cap = p.cap_rule;
   out->workspace_bytes = bytes;

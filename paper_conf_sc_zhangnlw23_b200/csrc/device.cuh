@@ -116,6 +116,7 @@ struct alignas(128) RowState {
   int src1;                      // source of the next pass: 0 = input row L, s + 1 = buffer slot s
   int win_state;                 // sample-guided window: 0 off, 1 window holds the K-th key, 2 failed
   unsigned long long win_lo, win_hi;  // window [lo, hi] of codes chosen from the sample
+  unsigned long long win_nmin, win_max;  // ~min and max code of the window members (atomicMax)
 };
 
 template <typename T>

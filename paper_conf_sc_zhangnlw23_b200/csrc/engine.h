@@ -21,6 +21,7 @@ struct SelectArgs {
   int ctas_per_row = 0;
   int cluster_size = 0;
   int window = 0;                   // sample-guided window: 0 auto, 1 on, -1 off
+  int tma = 0;                      // bulk-copy streaming: 0 auto, 1 on, -1 off
   int64_t* trace = nullptr;
   void* const* events = nullptr;    // optional cudaEvent_t[n_events] recorded around launches
   int n_events = 0;
@@ -39,6 +40,8 @@ struct Plan {
   int csize;         // CTAs per cluster (cluster engine)
   int max_clusters;  // cluster engine: clusters the workspace has candidate buffers for
   int nsamp;         // grid engine: samples per row for the sample-guided window (0 = off)
+  int tail;          // grid engine: finish after the window pass with one cluster-engine launch
+  int tma;           // grid engine: stream rows through bulk-copy (TMA) shared rings, 1 CTA/SM
   size_t off_state, off_hist, off_bcode, off_bidx, off_samp, bytes;
 };
 

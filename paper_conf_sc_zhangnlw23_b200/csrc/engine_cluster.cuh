@@ -38,11 +38,13 @@ struct ClusterParams {
   int P, IB;
   void* out_vals;
   int64_t* out_idx;
-  unsigned long long* counters;  // per row: out_count, buf_count[2], error (zeroed by the launcher)
-  void* bcode;                   // per cluster: 2 x cap_alloc codes
-  void* bidx;                    // per cluster: 2 x cap_alloc indices
+  RowState* st;  // per row (same workspace layout as the grid engine; counters, window outcome)
+  void* bcode;   // per row: 2 x cap_alloc codes   (slot-major: [slot][row][cap])
+  void* bidx;    // per row: 2 x cap_alloc indices
   int64_t cap_rule, cap_alloc;
   int nclusters;
+  int tail;      // 1: continue rows after the grid engine's window pass
+  int64_t* timing;  // optional: per CTA [globaltimer at start, at end, rows done, passes run]
 };
 
 struct ClusterShared {
@@ -53,16 +55,18 @@ struct ClusterShared {
   ScanResult scan;
 };
 
+// The cluster engine keeps ONE histogram copy: its passes are short, so zeroing/merging copies
+// costs more than the same-bin serialisation they avoid.
 template <int KIND, typename IdxT, int DF, int DH, bool HASIDX>
 __device__ __forceinline__ unsigned long long cluster_pass(PassCtx<typename KT<KIND>::U, IdxT>& c) {
-  return run_pass<KIND, IdxT, DF, DH, HASIDX, kCBlock>(c);
+  return run_pass<KIND, IdxT, DF, DH, HASIDX, kCBlock, 1>(c);
 }
 
 template <int KIND, typename IdxT, bool HASIDX>
 __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams p) {
   using U = typename KT<KIND>::U;
-  constexpr int HC = hist_copies<KIND, IdxT, 1>();
-  extern __shared__ unsigned sh_hist[];  // kMaxBins * HC
+  constexpr int HC = 1;
+  extern __shared__ unsigned sh_hist[];  // kHistSlots counters
   __shared__ WarpQ<U, IdxT> sh_oq[kCWarps];
   __shared__ WarpQ<U, IdxT> sh_bq[kCWarps];
   __shared__ ClusterShared cs;
@@ -78,47 +82,72 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
   const unsigned long long kk = (unsigned long long)p.k;
   const unsigned long long cap = (unsigned long long)p.cap_rule;
 
-  U* const bcode0 = (U*)p.bcode + (size_t)cid * 2 * p.cap_alloc;
-  IdxT* const bidx0 = (IdxT*)p.bidx + (size_t)cid * 2 * p.cap_alloc;
+  if (p.tail) pdl_wait();  // the window pass (previous launch) has finished every row
+  unsigned long long t_start = 0;
+  int n_rows = 0, n_passes = 0;
+  if (p.timing && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
 
   for (int64_t row = cid; row < p.batch; row += p.nclusters) {
-    unsigned long long* ctr = p.counters + row * 4;
+    RowState* st = p.st + row;
     unsigned long long K = kk, C = N, Cp = N, tcode = 0, tidx = 0;
-    int stop1 = 0;
-    for (int q = 0; q <= p.P; ++q) {
+    int stop1 = 0, src1 = 0;  // src1: 0 = the input row L, s + 1 = candidate buffer slot s
+    int q0 = 0;
+    if (p.tail && st->win_state == 1) {  // window held the K-th key: finish on the window buffer
+      K = st->K;
+      C = st->C;
+      Cp = st->C;
+      src1 = st->src1;
+      // Every window member lies in [wmin, wmax]: a key digit on which wmin and wmax (and all higher
+      // digits) agree has a one-bin histogram (j = that digit, K and C unchanged), so its pass is
+      // skipped — the paper's adaptivity applied to the digits.
+      const unsigned long long wmin = ~st->win_nmin, wmax = st->win_max;
+      const int pc = code_passes(KT<KIND>::R);
+      while (q0 < pc) {
+        const Digit d = digit_of(q0, KT<KIND>::R, p.IB);
+        if ((wmin >> d.shift) != (wmax >> d.shift)) break;
+        tcode |= ((wmin >> d.shift) & ((1ull << d.width) - 1ull)) << d.shift;
+        ++q0;
+      }
+    }
+    for (int q = q0; q <= p.P; ++q) {
       if (stop1 != 0 && stop1 - 1 < q - 1) break;
       const int DF = q == 0 ? 0 : (digit_of(q - 1, KT<KIND>::R, p.IB).is_idx ? 2 : 1);
       const int DH = q == p.P ? 0 : (digit_of(q, KT<KIND>::R, p.IB).is_idx ? 2 : 1);
+      const int sslot = (src1 == 1) ? 1 : 0;
       PassCtx<U, IdxT> c;
       c.q = q;
       c.emit_all = (DF != 0) && ((stop1 != 0 && stop1 - 1 == q - 1) || DH == 0);
       c.do_hist = (DH != 0) && !c.emit_all;
-      c.srcL = (DF == 0) || (Cp > cap);
-      c.store = c.do_hist && (DF != 0) && (C <= cap);
+      c.srcL = (src1 == 0);                                      // Alg1 L7-8
+      c.store = c.do_hist && (DF != 0) && (C <= cap);           // Alg1 L17
       c.sel_min = sel_min;
       c.reverse = (q & 1) != 0;
       c.dh = digit_of(q, KT<KIND>::R, p.IB);
       c.df = digit_of(DF != 0 ? q - 1 : 0, KT<KIND>::R, p.IB);
       c.tcode = tcode;
       c.tidx = tidx;
+      c.lo = 0;
+      c.wnmin = nullptr;
+      c.wmax = nullptr;
+      c.span1 = 0;
       c.rowp = (const U*)p.keys + row * p.len;
       c.rowi = HASIDX ? p.in_idx + row * p.len : nullptr;
       c.len = p.len;
       c.slice = crank;
       c.nslices = CS;
-      const int islot = (q - 1) & 1;
-      c.bcin = bcode0 + (size_t)islot * p.cap_alloc;
-      c.biin = bidx0 + (size_t)islot * p.cap_alloc;
-      c.nbuf = (DF != 0 && !c.srcL) ? __ldcg(&ctr[1 + islot]) : 0ull;
+      const int islot = src1 > 0 ? src1 - 1 : 0;
+      c.bcin = (const U*)p.bcode + ((size_t)islot * p.batch + row) * p.cap_alloc;
+      c.biin = (const IdxT*)p.bidx + ((size_t)islot * p.batch + row) * p.cap_alloc;
+      c.nbuf = (src1 > 0) ? __ldcg(&st->buf_count[islot]) : 0ull;
       c.ov = (U*)p.out_vals + row * p.k;
       c.oi = p.out_idx + row * p.k;
-      c.outc = &ctr[0];
+      c.outc = &st->out_count;
       c.kk = kk;
-      c.bco = bcode0 + (size_t)(q & 1) * p.cap_alloc;
-      c.bio = bidx0 + (size_t)(q & 1) * p.cap_alloc;
-      c.bufc = &ctr[1 + (q & 1)];
+      c.bco = (U*)p.bcode + ((size_t)sslot * p.batch + row) * p.cap_alloc;
+      c.bio = (IdxT*)p.bidx + ((size_t)sslot * p.batch + row) * p.cap_alloc;
+      c.bufc = &st->buf_count[sslot];
       c.capa = (unsigned long long)p.cap_alloc;
-      c.err = (unsigned*)&ctr[3];
+      c.err = &st->error;
       c.hist = sh_hist;
       c.oq = &sh_oq[warp];
       c.bq = &sh_bq[warp];
@@ -134,61 +163,71 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
         case 2 * 3 + 2: cluster_pass<KIND, IdxT, 2, 2, HASIDX>(c); break;
         default: cluster_pass<KIND, IdxT, 2, 0, HASIDX>(c); break;
       }
+      ++n_passes;
       if (!hist_on) break;  // emit-all pass: the row is complete
 
-      // ---- cluster-wide histogram merge + scan (replaces the last-block scan) ----
-      cl.sync();  // (B) every CTA's histogram and appends are complete
-      const int hc = (DF == 0) ? 1 : HC;   // copies used by this pass
+      // ---- histogram merge + scan (replaces the last-block scan) ----
       const int nb = 1 << c.dh.width;
-      const int seg = (nb + CS - 1) / CS;
-      const int b0 = crank * seg;
-      unsigned long long mytot = 0;
-      for (int i = tid; i < seg; i += kCBlock) {
-        const int b = b0 + i;
-        unsigned v = 0;
-        if (b < nb) {
-          for (int r = 0; r < CS; ++r) {
-            const unsigned* rh = cl.map_shared_rank(sh_hist, r);
-            for (int h = 0; h < hc; ++h) v += rh[b * hc + h];
-          }
-        }
-        sh_seg[i] = v;
-        mytot += v;
-      }
-      // block reduction of mytot
-      {
-        unsigned long long tot;
-        (void)block_exclusive_scan<kCBlock>(mytot, cs.tmp, tot);
-        if (tid == 0) {
-          for (int r = 0; r < CS; ++r) cl.map_shared_rank(&cs, r)->segtot[crank] = tot;
-        }
-      }
-      cl.sync();  // (C) all segment totals published; all remote reads of sh_hist done
-      unsigned long long before_seg = 0;
-      int owner = -1;
-      {
-        unsigned long long run = 0;
-        for (int r = 0; r < CS; ++r) {
-          const unsigned long long t = cs.segtot[r];
-          if (owner < 0 && run < K && run + t >= K) { owner = r; before_seg = run; }
-          run += t;
-        }
-      }
-      if (crank == owner) {
-        const unsigned long long Kseg = K - before_seg;
+      if (CS == 1) {
+        // one CTA per row: its histogram is the row's; scan it in place
+        __syncthreads();
         const ScanResult r = scan_choose<kCBlock>(
-            [&](int b) { return (unsigned long long)sh_seg[b]; }, seg, Kseg, cs.tmp, &cs.scan);
+            [&](int b) { return (unsigned long long)sh_hist[b]; }, nb, K, cs.tmp, &cs.scan);
         if (tid == 0) {
+          cs.res_j = r.j;
+          cs.res_before = r.before;
+          cs.res_cnt = r.cnt;
+        }
+        if (c.store) src1 = sslot + 1;  // the buffer this pass wrote feeds the next one
+        if (tid == 0) st->buf_count[src1 == 1 ? 1 : 0] = 0;  // next pass's output buffer
+        __syncthreads();
+      } else {
+        cl.sync();  // (B) every CTA's histogram and appends are complete
+        // CTA r owns bins [r*seg, (r+1)*seg): sum them over the cluster (all DSMEM loads in flight)
+        const int seg = (nb + CS - 1) / CS;
+        const int b0 = crank * seg;
+        for (int i = tid; i < seg; i += kCBlock) sh_seg[i] = 0;
+        __syncthreads();
+        const int pairs = seg * CS;
+        for (int pr = tid; pr < pairs; pr += kCBlock) {
+          const int b = pr % seg, rr = pr / seg;
+          const unsigned v = (b0 + b < nb) ? cl.map_shared_rank(sh_hist, rr)[b0 + b] : 0u;
+          if (v) atomicAdd(&sh_seg[b], v);
+        }
+        __syncthreads();
+        unsigned long long mytot = 0;
+        for (int i = tid; i < seg; i += kCBlock) mytot += sh_seg[i];
+        {
+          unsigned long long tot;
+          (void)block_exclusive_scan<kCBlock>(mytot, cs.tmp, tot);
+          if (tid < CS) cl.map_shared_rank(&cs, tid)->segtot[crank] = tot;
+        }
+        if (c.store) src1 = sslot + 1;
+        if (crank == 0 && tid == 0) st->buf_count[src1 == 1 ? 1 : 0] = 0;  // next pass's output buffer
+        cl.sync();  // (C) segment totals published; remote reads of sh_hist done
+        // every CTA finds the owner segment and scans the owner's merged bins (DSMEM) itself:
+        // identical result everywhere, no broadcast barrier
+        unsigned long long before_seg = 0;
+        int owner = 0;
+        {
+          unsigned long long run = 0;
+          bool found = false;
           for (int rr = 0; rr < CS; ++rr) {
-            ClusterShared* o = cl.map_shared_rank(&cs, rr);
-            o->res_j = (unsigned)(b0 + r.j);
-            o->res_before = before_seg + r.before;
-            o->res_cnt = r.cnt;
+            const unsigned long long t = cs.segtot[rr];
+            if (!found && run < K && run + t >= K) { owner = rr; before_seg = run; found = true; }
+            run += t;
           }
         }
+        const unsigned* oseg = cl.map_shared_rank(sh_seg, owner);
+        const ScanResult r = scan_choose<kCBlock>(
+            [&](int b) { return (unsigned long long)oseg[b]; }, seg, K - before_seg, cs.tmp, &cs.scan);
+        if (tid == 0) {
+          cs.res_j = (unsigned)(owner * seg + r.j);
+          cs.res_before = before_seg + r.before;
+          cs.res_cnt = r.cnt;
+        }
+        __syncthreads();
       }
-      if (crank == 0 && tid == 0) ctr[1 + ((q + 1) & 1)] = 0;  // buffer slot of pass q+1
-      cl.sync();  // (D) result visible everywhere
       const unsigned j = cs.res_j;
       const unsigned long long newK = K - cs.res_before, newC = cs.res_cnt;   // Alg1 L26-28
       Cp = C;
@@ -199,6 +238,13 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
       if (newK == newC) stop1 = q + 1;                                       // early stop
     }
     cl.sync();  // the cluster finishes the row before its buffers are reused
+    ++n_rows;
+  }
+  if (p.timing && tid == 0) {
+    unsigned long long t_end;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
+    int64_t* t = p.timing + (int64_t)blockIdx.x * 4;
+    t[0] = (int64_t)t_start; t[1] = (int64_t)t_end; t[2] = n_rows; t[3] = n_passes;
   }
 }
 
@@ -207,16 +253,19 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
 namespace airtopk {
 
 template <int KIND, typename IdxT, bool HASIDX>
-cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t s) {
+cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t s, int tail) {
   auto kern = cluster_kernel<KIND, IdxT, HASIDX>;
-  constexpr size_t smem = (size_t)kHistSlots * 4 * hist_copies<KIND, IdxT, 1>();
+  constexpr size_t smem = (size_t)kHistSlots * 4;
   static const cudaError_t attr1 = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   static const cudaError_t attr2 = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
   if (attr1 != cudaSuccess) return attr1;
   if (attr2 != cudaSuccess) return attr2;
   char* base = (char*)ws;
-  cudaError_t e = cudaMemsetAsync(base + pl.off_state, 0, (size_t)a.batch * 32, s);
-  if (e != cudaSuccess) return e;
+  cudaError_t e = cudaSuccess;
+  if (!tail) {  // standalone: fresh row states (the tail mode continues the grid engine's)
+    e = cudaMemsetAsync(base + pl.off_state, 0, pl.off_hist - pl.off_state, s);
+    if (e != cudaSuccess) return e;
+  }
   ClusterParams p;
   p.keys = a.keys;
   p.in_idx = a.in_idx;
@@ -228,45 +277,49 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   p.IB = pl.IB;
   p.out_vals = a.out_vals;
   p.out_idx = a.out_idx;
-  p.counters = (unsigned long long*)(base + pl.off_state);
+  p.st = (RowState*)(base + pl.off_state);
   p.bcode = base + pl.off_bcode;
   p.bidx = base + pl.off_bidx;
   p.cap_rule = pl.cap_rule;
   p.cap_alloc = pl.cap_alloc;
+  p.tail = tail;
+  p.timing = a.trace;  // cluster engine: the trace buffer receives per-CTA timing instead
 
   cudaLaunchConfig_t cfg = {};
-  cudaLaunchAttribute at[1];
+  cudaLaunchAttribute at[2];
   at[0].id = cudaLaunchAttributeClusterDimension;
   at[0].val.clusterDim.x = pl.csize;
   at[0].val.clusterDim.y = 1;
   at[0].val.clusterDim.z = 1;
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.blockDim = dim3(kCBlock, 1, 1);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
   cfg.attrs = at;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = tail ? 2 : 1;
   cfg.gridDim = dim3((unsigned)pl.csize, 1, 1);
   int maxc = 0;
   e = cudaOccupancyMaxActiveClusters(&maxc, kern, &cfg);
   if (e != cudaSuccess) return e;
   if (maxc < 1) return cudaErrorInvalidConfiguration;
-  const int64_t ncl = std::min<int64_t>({a.batch, (int64_t)maxc, (int64_t)pl.max_clusters});
+  const int64_t ncl = std::min<int64_t>(a.batch, (int64_t)maxc);
   p.nclusters = (int)ncl;
   cfg.gridDim = dim3((unsigned)(ncl * pl.csize), 1, 1);
-  if (a.events && a.n_events > 0) cudaEventRecord((cudaEvent_t)a.events[0], s);
+  if (!tail && a.events && a.n_events > 0) cudaEventRecord((cudaEvent_t)a.events[0], s);
   e = cudaLaunchKernelEx(&cfg, kern, p);
-  if (a.events && a.n_events > 1) cudaEventRecord((cudaEvent_t)a.events[1], s);
+  if (!tail && a.events && a.n_events > 1) cudaEventRecord((cudaEvent_t)a.events[1], s);
   return e;
 }
 
 template <int KIND>
-cudaError_t launch_cluster_kind(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t s) {
-  if (a.in_idx) return launch_cluster_t<KIND, uint64_t, true>(a, pl, ws, s);
-  if (pl.idx64) return launch_cluster_t<KIND, uint64_t, false>(a, pl, ws, s);
-  return launch_cluster_t<KIND, uint32_t, false>(a, pl, ws, s);
+cudaError_t launch_cluster_kind(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t s, int tail) {
+  if (a.in_idx) return launch_cluster_t<KIND, uint64_t, true>(a, pl, ws, s, tail);
+  if (pl.idx64) return launch_cluster_t<KIND, uint64_t, false>(a, pl, ws, s, tail);
+  return launch_cluster_t<KIND, uint32_t, false>(a, pl, ws, s, tail);
 }
 
 #define AIRTOPK_INSTANTIATE_CLUSTER(KIND) \
-  template cudaError_t launch_cluster_kind<KIND>(const SelectArgs&, const Plan&, void*, cudaStream_t);
+  template cudaError_t launch_cluster_kind<KIND>(const SelectArgs&, const Plan&, void*, cudaStream_t, int);
 
 }  // namespace airtopk

@@ -6,17 +6,17 @@
 
 namespace airtopk {
 
-extern template cudaError_t launch_grid_kind<K_F32>(const SelectArgs&, const Plan&, const GridParams&, cudaStream_t);
-extern template cudaError_t launch_grid_kind<K_F16>(const SelectArgs&, const Plan&, const GridParams&, cudaStream_t);
-extern template cudaError_t launch_grid_kind<K_BF16>(const SelectArgs&, const Plan&, const GridParams&, cudaStream_t);
-extern template cudaError_t launch_grid_kind<K_F64>(const SelectArgs&, const Plan&, const GridParams&, cudaStream_t);
-extern template cudaError_t launch_grid_kind<K_U32>(const SelectArgs&, const Plan&, const GridParams&, cudaStream_t);
+extern template cudaError_t launch_grid_kind<K_F32>(const SelectArgs&, const Plan&, const GridParams&, void*, cudaStream_t);
+extern template cudaError_t launch_grid_kind<K_F16>(const SelectArgs&, const Plan&, const GridParams&, void*, cudaStream_t);
+extern template cudaError_t launch_grid_kind<K_BF16>(const SelectArgs&, const Plan&, const GridParams&, void*, cudaStream_t);
+extern template cudaError_t launch_grid_kind<K_F64>(const SelectArgs&, const Plan&, const GridParams&, void*, cudaStream_t);
+extern template cudaError_t launch_grid_kind<K_U32>(const SelectArgs&, const Plan&, const GridParams&, void*, cudaStream_t);
 int grid_occupancy_f32(int idx64);
-extern template cudaError_t launch_cluster_kind<K_F32>(const SelectArgs&, const Plan&, void*, cudaStream_t);
-extern template cudaError_t launch_cluster_kind<K_F16>(const SelectArgs&, const Plan&, void*, cudaStream_t);
-extern template cudaError_t launch_cluster_kind<K_BF16>(const SelectArgs&, const Plan&, void*, cudaStream_t);
-extern template cudaError_t launch_cluster_kind<K_F64>(const SelectArgs&, const Plan&, void*, cudaStream_t);
-extern template cudaError_t launch_cluster_kind<K_U32>(const SelectArgs&, const Plan&, void*, cudaStream_t);
+extern template cudaError_t launch_cluster_kind<K_F32>(const SelectArgs&, const Plan&, void*, cudaStream_t, int);
+extern template cudaError_t launch_cluster_kind<K_F16>(const SelectArgs&, const Plan&, void*, cudaStream_t, int);
+extern template cudaError_t launch_cluster_kind<K_BF16>(const SelectArgs&, const Plan&, void*, cudaStream_t, int);
+extern template cudaError_t launch_cluster_kind<K_F64>(const SelectArgs&, const Plan&, void*, cudaStream_t, int);
+extern template cudaError_t launch_cluster_kind<K_U32>(const SelectArgs&, const Plan&, void*, cudaStream_t, int);
 
 // K == N ("a trivial case"): every element is a result, in index order.
 template <typename U>
@@ -60,22 +60,22 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t
   gp.trace = a.trace;
   gp.samp = base + pl.off_samp;
   switch (a.kind) {
-    case K_F32: return launch_grid_kind<K_F32>(a, pl, gp, s);
-    case K_F16: return launch_grid_kind<K_F16>(a, pl, gp, s);
-    case K_BF16: return launch_grid_kind<K_BF16>(a, pl, gp, s);
-    case K_F64: return launch_grid_kind<K_F64>(a, pl, gp, s);
-    case K_U32: return launch_grid_kind<K_U32>(a, pl, gp, s);
+    case K_F32: return launch_grid_kind<K_F32>(a, pl, gp, ws, s);
+    case K_F16: return launch_grid_kind<K_F16>(a, pl, gp, ws, s);
+    case K_BF16: return launch_grid_kind<K_BF16>(a, pl, gp, ws, s);
+    case K_F64: return launch_grid_kind<K_F64>(a, pl, gp, ws, s);
+    case K_U32: return launch_grid_kind<K_U32>(a, pl, gp, ws, s);
   }
   return cudaErrorInvalidValue;
 }
 
 cudaError_t run_cluster(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t s) {
   switch (a.kind) {
-    case K_F32: return launch_cluster_kind<K_F32>(a, pl, ws, s);
-    case K_F16: return launch_cluster_kind<K_F16>(a, pl, ws, s);
-    case K_BF16: return launch_cluster_kind<K_BF16>(a, pl, ws, s);
-    case K_F64: return launch_cluster_kind<K_F64>(a, pl, ws, s);
-    case K_U32: return launch_cluster_kind<K_U32>(a, pl, ws, s);
+    case K_F32: return launch_cluster_kind<K_F32>(a, pl, ws, s, 0);
+    case K_F16: return launch_cluster_kind<K_F16>(a, pl, ws, s, 0);
+    case K_BF16: return launch_cluster_kind<K_BF16>(a, pl, ws, s, 0);
+    case K_F64: return launch_cluster_kind<K_F64>(a, pl, ws, s, 0);
+    case K_U32: return launch_cluster_kind<K_U32>(a, pl, ws, s, 0);
   }
   return cudaErrorInvalidValue;
 }

@@ -66,13 +66,24 @@ struct GridParams {
 
 constexpr int kBlock = 512;
 constexpr int kWarps = kBlock / 32;
-constexpr int kMinBlocks = 3;
-constexpr int kMinBlocksFilter = AIRTOPK_SLOW_REG ? 2 : 3;
+
+// dynamic shared memory of a pass kernel: [histogram copies][TMA warp rings][ring mbarriers]
+template <int HC>
+constexpr size_t tma_ring_offset() { return ((size_t)kHistSlots * 4 * HC + 127) / 128 * 128; }
+template <int KIND>
+constexpr size_t tma_ring_bytes() { return (size_t)kWarps * kTmaStages * 32 * kUnroll * 16; }
+#ifndef AIRTOPK_MINB
+#define AIRTOPK_MINB 3
+#endif
+constexpr int kMinBlocks = AIRTOPK_MINB;
+constexpr int kMinBlocksFilter = AIRTOPK_SLOW_REG ? 2 : AIRTOPK_MINB;
 
 // Kernel q of the select. DF/DH: digit filtered / histogrammed (passes.cuh). DF == 3 is the
 // sample-guided window pass (q = 0); `redo` = the pass-0 histogram re-run over the window buffer.
-template <int KIND, typename IdxT, int DF, int DH, bool HASIDX>
-__global__ void __launch_bounds__(kBlock, (DF == 0 ? kMinBlocks : kMinBlocksFilter))
+// TMA: the input row is streamed through per-warp shared rings by the bulk-copy engine (1 CTA/SM,
+// DESIGN.md "Kernels"); otherwise 4 x 16-byte register loads per thread (3 CTAs/SM).
+template <int KIND, typename IdxT, int DF, int DH, bool HASIDX, bool TMA = false>
+__global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMinBlocksFilter))
     pass_kernel(const GridParams p, const int q, const int redo) {
   using U = typename KT<KIND>::U;
   using CountT = std::conditional_t<sizeof(IdxT) == 8, unsigned long long, unsigned>;
@@ -117,6 +128,8 @@ __global__ void __launch_bounds__(kBlock, (DF == 0 ? kMinBlocks : kMinBlocksFilt
   c.df = digit_of(FILTER ? q - 1 : 0, KT<KIND>::R, p.IB);
   c.tcode = FILTER ? st->tcode : 0ull;
   c.tidx = FILTER ? st->tidx : 0ull;
+  c.wnmin = &st->win_nmin;
+  c.wmax = &st->win_max;
   c.lo = (win_state == 1) ? st->win_lo : 0ull;
   c.span1 = (win_state == 1) ? st->win_hi - st->win_lo + 1ull : 0ull;
   c.rowp = (const U*)p.keys + row * p.len;
@@ -138,6 +151,8 @@ __global__ void __launch_bounds__(kBlock, (DF == 0 ? kMinBlocks : kMinBlocksFilt
   c.capa = (unsigned long long)p.cap_alloc;
   c.err = &st->error;
   c.hist = sh_hist;
+  c.ring = smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>();
+  c.bars = c.ring + (unsigned)tma_ring_bytes<KIND>();
   c.oq = &sh_oq[HAS_Q ? warp : 0];
   c.bq = &sh_bq[(HAS_Q && (DH != 0 || DF == 3)) ? warp : 0];
 
@@ -147,7 +162,7 @@ __global__ void __launch_bounds__(kBlock, (DF == 0 ? kMinBlocks : kMinBlocksFilt
     __syncthreads();
   }
 
-  const unsigned long long nread = run_pass<KIND, IdxT, DF, DH, HASIDX, kBlock>(c);
+  const unsigned long long nread = run_pass<KIND, IdxT, DF, DH, HASIDX, kBlock, 0, TMA>(c);
 
   if constexpr (DF == 3) {
     // ---- window pass: the last CTA validates the window. R results below lo, Wn members inside;
@@ -235,52 +250,62 @@ __global__ void __launch_bounds__(kBlock, (DF == 0 ? kMinBlocks : kMinBlocksFilt
 constexpr int kSampleBlock = 1024;
 constexpr int kMaxSamples = 16384;
 
+// MSD radix select (8-bit digits) of the elements of ranks r1 <= r2 (0-based) among a[0..n) in shared
+// memory, both at once: one pass over the data builds the digit histograms of both prefixes (a single
+// histogram while the two prefixes coincide); warps 0 and 1 scan them (8 bins per lane + shuffles).
 template <typename W>
-__device__ W block_select_rank(const W* a, int n, int rank, int bits, unsigned* hist, W* shw) {
-  // MSD radix select (8-bit digits) of the element of rank `rank` (0-based) among a[0..n) in shared
-  // memory; the 256-bin scan is done by warp 0 (8 bins per lane + shuffle scan).
-  W prefix = 0, pmask = 0;
-  int rk = rank;
-  const int lane = threadIdx.x & 31;
+__device__ void block_select_two(const W* a, int n, int r1, int r2, int bits, unsigned* hist /*512*/,
+                                 W* shw /*4*/, W& out1, W& out2) {
+  W p1 = 0, p2 = 0, mask = 0;
+  int k1 = r1, k2 = r2;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   for (int hi = bits; hi > 0; hi -= 8) {
     const int w = hi < 8 ? hi : 8, sh = hi - w;
-    for (int i = threadIdx.x; i < 256; i += blockDim.x) hist[i] = 0;
+    const bool same = (p1 == p2);
+    for (int i = threadIdx.x; i < 512; i += blockDim.x) hist[i] = 0;
     __syncthreads();
+#pragma unroll 4
     for (int i = threadIdx.x; i < n; i += blockDim.x) {
       const W v = a[i];
-      if ((v & pmask) == prefix) atomicAdd(&hist[(unsigned)(v >> sh) & 255u], 1u);
+      const unsigned d = (unsigned)(v >> sh) & 255u;
+      if ((v & mask) == p1) atomicAdd(&hist[d], 1u);
+      if (!same && (v & mask) == p2) atomicAdd(&hist[256 + d], 1u);
     }
     __syncthreads();
-    if (threadIdx.x < 32) {
+    if (warp < 2) {
+      const unsigned* h = hist + ((warp == 1 && !same) ? 256 : 0);
+      const int rk = (warp == 0) ? k1 : k2;
       unsigned c[8], tot = 0;
 #pragma unroll
-      for (int t = 0; t < 8; ++t) { c[t] = hist[lane * 8 + t]; tot += c[t]; }
+      for (int t = 0; t < 8; ++t) { c[t] = h[lane * 8 + t]; tot += c[t]; }
       unsigned incl = tot;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const unsigned y = __shfl_up_sync(kFull, incl, o);
         if (lane >= o) incl += y;
       }
-      unsigned run = incl - tot;  // bins before this lane's 8
+      unsigned run = incl - tot;
       if (run <= (unsigned)rk && (unsigned)rk < incl) {
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
           if (run <= (unsigned)rk && (unsigned)rk < run + c[t]) {
-            shw[0] = (W)(lane * 8 + t);
-            shw[1] = (W)run;
+            shw[warp * 2] = (W)(lane * 8 + t);
+            shw[warp * 2 + 1] = (W)run;
           }
           run += c[t];
         }
       }
     }
     __syncthreads();
-    const W d = shw[0];
-    rk -= (int)shw[1];
-    prefix |= d << sh;
-    pmask |= (W)((1u << w) - 1u) << sh;
+    p1 |= shw[0] << sh;
+    k1 -= (int)shw[1];
+    p2 |= shw[2] << sh;
+    k2 -= (int)shw[3];
+    mask |= (W)((1u << w) - 1u) << sh;
     __syncthreads();
   }
-  return prefix;
+  out1 = p1;
+  out2 = p2;
 }
 
 constexpr int kSampleCTAs = 16;  // CTAs per row issuing the scattered sample loads (one SM cannot
@@ -292,8 +317,8 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
   extern __shared__ __align__(16) unsigned char sample_smem[];
   W* codes = (W*)sample_smem;  // nsamp codes (last CTA only)
-  __shared__ unsigned hist[256];
-  __shared__ W shw[2];
+  __shared__ unsigned hist[512];
+  __shared__ W shw[4];
   __shared__ int sh_last;
   const int64_t row = blockIdx.x / kSampleCTAs;
   const int part = blockIdx.x % kSampleCTAs;
@@ -303,20 +328,23 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
   const U* rowp = (const U*)p.keys + row * p.len;
   W* samp = (W*)p.samp + row * (int64_t)nsamp;
   const U xmask = p.sel_min ? (U)0 : (U)~(U)0;
-  const int64_t stride = p.len / nsamp;
-  // phase 1: stratified samples s = part, part + 16, ... (all of this CTA's loads in flight at once)
+  // Samples come in runs of kRun consecutive elements (one 128-byte line for f32) at nsamp/kRun
+  // stratified positions: a DRAM line is fetched whole anyway, so this costs nsamp*4 bytes of traffic
+  // instead of nsamp*128. (Runs are independent draws for i.i.d. data; a row whose order defeats the
+  // estimate only triggers the fallback.)
+  constexpr int kRun = 32;
+  const int nruns = nsamp / kRun;
+  const int64_t stride = p.len / nruns;
+  // phase 1: this CTA's runs part, part + 16, ... (all loads in flight at once)
   {
     constexpr int PER = kMaxSamples / (kSampleBlock * kSampleCTAs);
-    W v[PER];
 #pragma unroll
     for (int t = 0; t < PER; ++t) {
-      const int s = (t * kSampleBlock + threadIdx.x) * kSampleCTAs + part;
-      v[t] = (s < nsamp) ? (W)to_code_x<KIND>(__ldg(rowp + (int64_t)s * stride + stride / 2), xmask) : (W)0;
-    }
-#pragma unroll
-    for (int t = 0; t < PER; ++t) {
-      const int s = (t * kSampleBlock + threadIdx.x) * kSampleCTAs + part;
-      if (s < nsamp) samp[s] = v[t];
+      const int slot = t * kSampleBlock + threadIdx.x;  // (run-in-part, lane)
+      const int run = (slot / kRun) * kSampleCTAs + part, e = slot % kRun;
+      const int s = run * kRun + e;
+      const int64_t pos = (int64_t)run * stride + (stride - kRun) / 2 + e;
+      if (run < nruns && pos < p.len) samp[s] = (W)to_code_x<KIND>(__ldg(rowp + pos), xmask);
     }
   }
   __threadfence();
@@ -326,21 +354,36 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
   if (!sh_last) return;
   __threadfence();
   // phase 2 (last CTA of the row): the window from the sample order statistics
-  for (int s = threadIdx.x; s < nsamp; s += blockDim.x) codes[s] = __ldcg(samp + s);
+  {
+    constexpr int PER = kMaxSamples / kSampleBlock;  // all L2 loads in flight at once
+    W v[PER];
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+      const int s = t * kSampleBlock + threadIdx.x;
+      v[t] = (s < nsamp) ? __ldcg(samp + s) : (W)0;
+    }
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+      const int s = t * kSampleBlock + threadIdx.x;
+      if (s < nsamp) codes[s] = v[t];
+    }
+  }
   __syncthreads();
   if (threadIdx.x == 0) st->ticket = 0;
-  // expected sample rank of the K-th key and a 3.5-sigma (+3) margin of the binomial sample count:
-  // a miss (probability < 1e-3) only costs the fallback, never exactness
+  // expected sample rank of the K-th key and a 4-sigma (+8) margin of the binomial sample count
+  // (measured sample counts are somewhat over-dispersed): a miss only costs the fallback, never
+  // exactness
   const double f = (double)p.k / (double)p.len;
   const double r = f * nsamp;
-  const double m = 3.5 * sqrt(r * (1.0 - f)) + 3.0;
+  const double m = 4.0 * sqrt(r * (1.0 - f)) + 8.0;
   const int rlo = (int)floor(r - m), rhi = (int)ceil(r + m);
   if (rhi >= nsamp - 1) {  // the window would hold most of the row: keep the paper's passes
     if (threadIdx.x == 0) st->win_state = 0;
     return;
   }
-  const W lo = (rlo <= 0) ? (W)0 : block_select_rank<W>(codes, nsamp, rlo, KT<KIND>::R, hist, shw);
-  const W hi = block_select_rank<W>(codes, nsamp, rhi, KT<KIND>::R, hist, shw);
+  W lo, hi;
+  block_select_two<W>(codes, nsamp, rlo > 0 ? rlo : 0, rhi, KT<KIND>::R, hist, shw, lo, hi);
+  if (rlo <= 0) lo = 0;  // no results below the window: everything up to hi is a candidate
   if (threadIdx.x == 0) {
     st->win_lo = lo;
     st->win_hi = hi;
@@ -373,22 +416,25 @@ struct Events {
   }
 };
 
-template <int KIND, typename IdxT, int DF, int DH>
+template <int KIND, typename IdxT, int DF, int DH, bool TMA = false>
 constexpr size_t hist_smem_bytes() {
-  return (size_t)kHistSlots * 4 * hist_copies<KIND, IdxT, DF>();
+  constexpr int HC = hist_copies<KIND, IdxT, DF>();
+  return TMA ? tma_ring_offset<HC>() + tma_ring_bytes<KIND>() + (size_t)kWarps * kTmaStages * 8
+             : (size_t)kHistSlots * 4 * HC;
 }
 
-template <int KIND, typename IdxT, int DF, int DH, bool HASIDX>
+template <int KIND, typename IdxT, int DF, int DH, bool HASIDX, bool TMA>
 cudaError_t launch_one(const GridParams& gp, unsigned grid, int q, int redo, cudaStream_t s) {
-  constexpr size_t smem = hist_smem_bytes<KIND, IdxT, DF, DH>();
-  static const cudaError_t attr = cudaFuncSetAttribute(pass_kernel<KIND, IdxT, DF, DH, HASIDX>,
+  constexpr size_t smem = hist_smem_bytes<KIND, IdxT, DF, DH, TMA>();
+  static const cudaError_t attr = cudaFuncSetAttribute(pass_kernel<KIND, IdxT, DF, DH, HASIDX, TMA>,
                                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (attr != cudaSuccess) return attr;
-  return launch_pdl(pass_kernel<KIND, IdxT, DF, DH, HASIDX>, dim3(grid), dim3(kBlock), smem, s, gp, q, redo);
+  return launch_pdl(pass_kernel<KIND, IdxT, DF, DH, HASIDX, TMA>, dim3(grid), dim3(kBlock), smem, s, gp, q, redo);
 }
 
-template <int KIND, typename IdxT, bool HASIDX>
-cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, const Events& ev, cudaStream_t s) {
+template <int KIND, typename IdxT, bool HASIDX, bool TMA = false>
+cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, const Events& ev, cudaStream_t s,
+                               bool window_only = false) {
   const unsigned grid = (unsigned)((long long)batch * gp.cpr);
   int ie = 0;
   ev.record(ie++, s);
@@ -402,9 +448,10 @@ cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, c
                                 (size_t)nsamp * sizeof(W), s, gp, nsamp);
     if (es != cudaSuccess) return es;
     ev.record(ie++, s);
-    cudaError_t e = launch_one<KIND, IdxT, 3, 0, HASIDX>(gp, grid, 0, 0, s);
+    cudaError_t e = launch_one<KIND, IdxT, 3, 0, HASIDX, TMA>(gp, grid, 0, 0, s);
     if (e != cudaSuccess) return e;
     ev.record(ie++, s);
+    if (window_only) return cudaGetLastError();
   }
   for (int q = 0; q <= gp.P; ++q) {
     const int DF = q == 0 ? 0 : (digit_of(q - 1, KT<KIND>::R, gp.IB).is_idx ? 2 : 1);
@@ -413,11 +460,11 @@ cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, c
     cudaError_t e;
     const int redo = (q == 0 && nsamp > 0) ? 1 : 0;
     switch (v) {
-      case 0 * 3 + 1: e = launch_one<KIND, IdxT, 0, 1, HASIDX>(gp, grid, q, redo, s); break;
-      case 1 * 3 + 1: e = launch_one<KIND, IdxT, 1, 1, HASIDX>(gp, grid, q, 0, s); break;
-      case 1 * 3 + 2: e = launch_one<KIND, IdxT, 1, 2, HASIDX>(gp, grid, q, 0, s); break;
-      case 2 * 3 + 2: e = launch_one<KIND, IdxT, 2, 2, HASIDX>(gp, grid, q, 0, s); break;
-      case 2 * 3 + 0: e = launch_one<KIND, IdxT, 2, 0, HASIDX>(gp, grid, q, 0, s); break;
+      case 0 * 3 + 1: e = launch_one<KIND, IdxT, 0, 1, HASIDX, TMA>(gp, grid, q, redo, s); break;
+      case 1 * 3 + 1: e = launch_one<KIND, IdxT, 1, 1, HASIDX, TMA>(gp, grid, q, 0, s); break;
+      case 1 * 3 + 2: e = launch_one<KIND, IdxT, 1, 2, HASIDX, TMA>(gp, grid, q, 0, s); break;
+      case 2 * 3 + 2: e = launch_one<KIND, IdxT, 2, 2, HASIDX, TMA>(gp, grid, q, 0, s); break;
+      case 2 * 3 + 0: e = launch_one<KIND, IdxT, 2, 0, HASIDX, TMA>(gp, grid, q, 0, s); break;
       default: return cudaErrorInvalidValue;
     }
     if (e != cudaSuccess) return e;
@@ -427,14 +474,25 @@ cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, c
 }
 
 template <int KIND>
-cudaError_t launch_grid_kind(const SelectArgs& a, const Plan& pl, const GridParams& gp, cudaStream_t s) {
+cudaError_t launch_cluster_kind(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t s, int tail);
+
+// Grid engine. With pl.tail the rows are finished after the window pass by ONE cluster-engine launch
+// over the (small) window buffers instead of P+1 grid launches.
+template <int KIND>
+cudaError_t launch_grid_kind(const SelectArgs& a, const Plan& pl, const GridParams& gp, void* ws, cudaStream_t s) {
   const Events ev{a.events, a.n_events};
   if (a.in_idx) return launch_grid_passes<KIND, uint64_t, true>(gp, a.batch, 0, ev, s);
-  if (pl.idx64) return launch_grid_passes<KIND, uint64_t, false>(gp, a.batch, pl.nsamp, ev, s);
-  return launch_grid_passes<KIND, uint32_t, false>(gp, a.batch, pl.nsamp, ev, s);
+  cudaError_t e;
+  if (pl.idx64) e = launch_grid_passes<KIND, uint64_t, false>(gp, a.batch, pl.nsamp, ev, s, pl.tail != 0);
+  else if (pl.tma) e = launch_grid_passes<KIND, uint32_t, false, true>(gp, a.batch, pl.nsamp, ev, s, pl.tail != 0);
+  else e = launch_grid_passes<KIND, uint32_t, false>(gp, a.batch, pl.nsamp, ev, s, pl.tail != 0);
+  if (e != cudaSuccess || !pl.tail) return e;
+  e = launch_cluster_kind<KIND>(a, pl, ws, s, 1);
+  ev.record(3, s);
+  return e;
 }
 
 #define AIRTOPK_INSTANTIATE_GRID(KIND) \
-  template cudaError_t launch_grid_kind<KIND>(const SelectArgs&, const Plan&, const GridParams&, cudaStream_t);
+  template cudaError_t launch_grid_kind<KIND>(const SelectArgs&, const Plan&, const GridParams&, void*, cudaStream_t);
 
 }  // namespace airtopk

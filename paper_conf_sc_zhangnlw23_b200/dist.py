@@ -58,9 +58,11 @@ def _all_gather(t, group):
         out = torch.empty((world,) + tuple(t.shape), dtype=t.dtype, device=t.device)
         dist.all_gather_into_tensor(out, t.contiguous(), group=group)
         return out
-    parts = [torch.empty_like(t) for _ in range(world)]
-    dist.all_gather(parts, t.contiguous(), group=group)
-    return torch.stack(parts)
+    # gloo (CPU tests, or the multi-rank self-test of bench.py): gather through host memory
+    tc = t.contiguous().cpu()
+    parts = [torch.empty_like(tc) for _ in range(world)]
+    dist.all_gather(parts, tc, group=group)
+    return torch.stack(parts).to(t.device)
 
 
 def select_split_row(x_shard, k: int, total_len: int, shard_offset: int, largest: bool = False, group=None,
@@ -77,7 +79,11 @@ def select_split_row(x_shard, k: int, total_len: int, shard_offset: int, largest
     gidx = i.reshape(-1).to(torch.int64) + shard_offset
     if kk < k:  # pad so every rank contributes exactly k candidates (they sort last, never selected)
         pad = k - kk
-        pv = torch.full((pad,), pad_bits(x_shard.dtype, largest), dtype=_bits_view(v).dtype, device=v.device)
+        bits = pad_bits(x_shard.dtype, largest)
+        width = 8 * v.element_size()
+        if bits >= 1 << (width - 1):  # as the signed integer of the same width
+            bits -= 1 << width
+        pv = torch.full((pad,), bits, dtype=_bits_view(v).dtype, device=v.device)
         v = torch.cat([v, pv.view(v.dtype)])
         rank = dist.get_rank(group)
         gidx = torch.cat([gidx, total_len + rank * k + torch.arange(pad, dtype=torch.int64, device=gidx.device)])

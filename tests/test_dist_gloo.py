@@ -96,6 +96,7 @@ def test_split_row_merge_and_row_sharding(world):
     if world == 3:
         # every shard shorter than K: padding candidates must never be selected
         cases.append(dict(kind="split", n=1000, k=600, dist="adversarial", m=30, largest=False))
+        cases.append(dict(kind="split", n=1000, k=600, dist="uniform", m=20, largest=True))
     _run(world, cases)
 
 

@@ -268,9 +268,13 @@ def test_cluster_engine_alpha(alpha):
 # ---------------------------------------------------------------- sample-guided window (NEXT #1)
 
 def _sample_positions(n):
-    ns = min(max(n // 256, 1024), 16384, n)
-    stride = n // ns
-    return np.arange(ns, dtype=np.int64) * stride + stride // 2
+    """The positions the sample kernel reads (runs of 32 at stratified offsets, see api.cu)."""
+    ns = min(max(n // 128, 4096), 16384)
+    ns = min(ns, n // 2) // 32 * 32
+    runs = ns // 32
+    stride = n // runs
+    base = np.arange(runs, dtype=np.int64) * stride + (stride - 32) // 2
+    return (base[:, None] + np.arange(32)[None, :]).reshape(-1)
 
 
 @pytest.mark.parametrize("window", [-1, 1])
@@ -283,8 +287,9 @@ def test_window_on_off(window, dist, m, k):
         assert_parity(x, "f32", k, sm, v, i)
 
 
+@pytest.mark.parametrize("engine", [0, 1])
 @pytest.mark.parametrize("case", ["high", "low", "ties"])
-def test_window_fallback(case):
+def test_window_fallback(case, engine):
     """Inputs built so the stratified sample misrepresents the row: the window pass must detect the
     miss (R >= K or K > R + W) and fall back to the paper's passes, exactly."""
     n = 1 << 20
@@ -301,8 +306,21 @@ def test_window_fallback(case):
         x[pos] = np.float32(2.0)
         ks = (1, len(pos) + 1, 700000)
     for k in ks:
-        v, i = gpu_select(x, "f32", k, True, window=1, engine=1)
+        v, i = gpu_select(x, "f32", k, True, window=1, engine=engine)
         assert_parity(x, "f32", k, True, v, i)
+
+
+@pytest.mark.parametrize("dist,batch,n,k", [("normal", 100, 1 << 20, 256), ("adversarial", 3, 1 << 22, 5000),
+                                            ("uniform", 7, 1 << 19, 1), ("uniform", 2, 1 << 21, 20000)])
+def test_window_tail(dist, batch, n, k):
+    """auto engine: window pass + one cluster-engine launch finishing every row (tail mode)"""
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    assert at.describe(torch.float32, batch, n, k)["launches"] == 3
+    x = _keys(dist, 33, batch, n)
+    for sm in (True, False):
+        v, i = gpu_select(x, "f32", k, sm)
+        assert_parity(x, "f32", k, sm, v, i)
 
 
 def test_window_describe():
@@ -312,3 +330,18 @@ def test_window_describe():
     assert d["engine"] == 1 and d["launches"] == d["passes"] + 3
     d = at.describe(torch.float32, 1, 1 << 30, 1 << 20, window=-1)
     assert d["launches"] == d["passes"] + 1
+
+
+# ---------------------------------------------------------------- bulk-copy (TMA) streaming vs register loads
+
+@pytest.mark.parametrize("tma", [-1, 1])
+@pytest.mark.parametrize("window", [-1, 1])
+@pytest.mark.parametrize("dist,m,batch,n,k,off", [("uniform", 20, 1, (1 << 22) + 77, 3000, 0),
+                                                  ("adversarial", 20, 2, 1 << 22, 40000, 1),
+                                                  ("normal", 20, 3, 999999, 17, 3),
+                                                  ("adversarial", 12, 1, 1 << 21, 1 << 20, 2)])
+def test_tma_streaming(tma, window, dist, m, batch, n, k, off):
+    x = _keys(dist, 44, batch, n, m)
+    for sm in (True, False):
+        v, i = gpu_select(x, "f32", k, sm, offset_elems=off, tma=tma, window=window, engine=1)
+        assert_parity(x, "f32", k, sm, v, i)
