@@ -83,6 +83,7 @@ Plan make_plan(const SelectArgs& a) {
     // costs <= 1/64 of the row's bytes; at least 4K samples keep the window small vs N/alpha
     int64_t ns = std::min<int64_t>(std::max<int64_t>(a.len / 128, 4096), 16384);
     ns = std::min<int64_t>(ns, a.len / 2) / 32 * 32;
+    if (key_bytes(a.kind) == 8) ns = std::min<int64_t>(ns, 8192);  // sample_kernel shared memory
     p.nsamp = ns >= 1024 ? (int)ns : 0;
   }
   p.off_samp = p.off_bidx + align_up((size_t)2 * a.batch * p.cap_alloc * isz, 256);

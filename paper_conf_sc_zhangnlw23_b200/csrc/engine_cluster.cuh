@@ -92,17 +92,23 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
     unsigned long long K = kk, C = N, Cp = N, tcode = 0, tidx = 0;
     int stop1 = 0, src1 = 0;  // src1: 0 = the input row L, s + 1 = candidate buffer slot s
     int q0 = 0;
-    if (p.tail && st->win_state == 1) {  // window held the K-th key: finish on the window buffer
+    if (p.tail && st->win_state == 1) {
+      // the window held the K-th key and the window pass already scanned pass 1 over the window
+      // buffer: continue from its state
       K = st->K;
       C = st->C;
-      Cp = st->C;
+      Cp = st->Cp;
       src1 = st->src1;
-      // Every window member lies in [wmin, wmax]: a key digit on which wmin and wmax (and all higher
-      // digits) agree has a one-bin histogram (j = that digit, K and C unchanged), so its pass is
-      // skipped — the paper's adaptivity applied to the digits.
+      tcode = st->tcode;
+      stop1 = st->stop1;
+      q0 = st->npass;
+      // Every window member lies in [wmin, wmax]: while all key bits above digit q agree between the
+      // two (so no result of an earlier digit is pending), pass q's histogram is a single bin (j = that
+      // digit, K and C unchanged) and the pass is skipped — the paper's adaptivity applied to the
+      // digits.
       const unsigned long long wmin = ~st->win_nmin, wmax = st->win_max;
       const int pc = code_passes(KT<KIND>::R);
-      while (q0 < pc) {
+      while (stop1 == 0 && q0 < pc) {
         const Digit d = digit_of(q0, KT<KIND>::R, p.IB);
         if ((wmin >> d.shift) != (wmax >> d.shift)) break;
         tcode |= ((wmin >> d.shift) & ((1ull << d.width) - 1ull)) << d.shift;

@@ -111,7 +111,8 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   if (FILTER && stop1 != 0 && stop1 - 1 < q - 1) return;  // finished by an earlier early stop
   const int win_state = (DF == 3 || (DF == 0 && redo)) ? st->win_state : 0;
   if (DF == 3 && win_state != 1) return;                   // no window: pass 0 will read L
-  const bool redo_buf = (DF == 0) && redo && (win_state == 1);  // pass 0 over the window buffer
+  if (DF == 0 && redo && win_state == 1) return;           // pass 0 was done by the window pass
+  const bool redo_buf = false;
   const int src1 = (FILTER || redo_buf) ? st->src1 : 0;    // Alg1 L7-8 (reading 6)
   const int sslot = (src1 == 1) ? 1 : 0;                   // candidate buffer this pass writes
   PassCtx<U, IdxT> c;
@@ -156,40 +157,13 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.oq = &sh_oq[HAS_Q ? warp : 0];
   c.bq = &sh_bq[(HAS_Q && (DH != 0 || DF == 3)) ? warp : 0];
 
-  const bool hist_on = c.do_hist || DF == 0;
+  const bool hist_on = c.do_hist || DF == 0 || DF == 3;
   if (hist_on) {
     for (int i = tid; i < kHistSlots * HC; i += kBlock) sh_hist[i] = 0;
     __syncthreads();
   }
 
   const unsigned long long nread = run_pass<KIND, IdxT, DF, DH, HASIDX, kBlock, 0, TMA>(c);
-
-  if constexpr (DF == 3) {
-    // ---- window pass: the last CTA validates the window. R results below lo, Wn members inside;
-    // the K-th key lies in the window iff R < K <= R + Wn (and the buffer did not overflow) ----
-    __threadfence();
-    __syncthreads();
-    if (tid == 0) sh_last = (atomicAdd(&st->ticket, 1u) == (unsigned)(p.cpr - 1));
-    __syncthreads();
-    if (!sh_last || tid != 0) return;
-    __threadfence();
-    const unsigned long long kk = (unsigned long long)p.k;
-    const unsigned long long R = __ldcg(c.outc), Wn = __ldcg(c.bufc);
-    if ((__ldcg(&st->error) & 2u) == 0 && R < kk && kk <= R + Wn) {
-      st->K = kk - R;  // a fresh select of K - R among the Wn window members (pass 0 runs on them)
-      st->C = Wn;
-      st->Cp = Wn;
-      st->src1 = sslot + 1;
-      st->buf_count[sslot == 1 ? 0 : 1] = 0;
-    } else {
-      st->win_state = 2;  // miss: pass 0 re-reads L and the paper's passes follow
-      st->out_count = 0;
-      st->buf_count[sslot] = 0;
-      st->error &= ~2u;
-    }
-    st->ticket = 0;
-    return;
-  }
 
   if (!hist_on) return;
 
@@ -214,12 +188,34 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   const unsigned long long kk = (unsigned long long)p.k;
   unsigned long long Kin = (FILTER || redo_buf) ? st->K : kk;
   unsigned long long Cin = Cprev;  // elements counted by this histogram
+  bool window_ok = false;
+  if constexpr (DF == 3) {
+    // ---- window pass: R results below lo, Wn members inside; the K-th key lies in the window iff
+    // R < K <= R + Wn (and the buffer did not overflow). Then the histogram just merged is pass 1's
+    // over the window buffer: a fresh select of K - R among the Wn members continues from it. ----
+    const unsigned long long R = __ldcg(c.outc), Wn = __ldcg(c.bufc);
+    window_ok = (__ldcg(&st->error) & 2u) == 0 && R < kk && kk <= R + Wn;
+    Kin = kk - R;
+    Cin = Wn;
+    if (!window_ok) {  // miss: discard, the redo launch re-runs the paper's pass 1 over L
+      for (int i = tid; i < kMaxBins; i += kBlock) gh[i] = 0;
+      if (tid == 0) {
+        st->win_state = 2;
+        st->out_count = 0;
+        st->buf_count[sslot] = 0;
+        st->error &= ~2u;
+        st->ticket = 0;
+      }
+      return;
+    }
+  }
   const ScanResult r = scan_choose<kBlock>(
       [&](int b) { return (unsigned long long)__ldcg(&gh[b]); }, nb, Kin, sh_tmp, &sh_res);
   CountT* gh2 = (CountT*)p.ghist + ((size_t)row * 2 + ((q + 1) & 1)) * kMaxBins;
   for (int i = tid; i < kMaxBins; i += kBlock) gh2[i] = 0;
   if (tid == 0) {
     int next_src1 = (c.store) ? sslot + 1 : src1;  // the buffer this pass wrote feeds the next one
+    if (DF == 3) st->Cp = Cin;
     {
       const unsigned long long newK = Kin - r.before, newC = r.cnt;   // Alg1 L26-28
       st->Cp = Cin;
@@ -250,34 +246,26 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
 constexpr int kSampleBlock = 1024;
 constexpr int kMaxSamples = 16384;
 
-// MSD radix select (8-bit digits) of the elements of ranks r1 <= r2 (0-based) among a[0..n) in shared
-// memory, both at once: one pass over the data builds the digit histograms of both prefixes (a single
-// histogram while the two prefixes coincide); warps 0 and 1 scan them (8 bins per lane + shuffles).
+// Rank select among a[0..n) in shared memory with 8-bit MSD digits, below a fixed prefix (bits above
+// `hi_bits` equal `prefix` under `mask`). The 256-bin scan is done by warp 0 (8 bins per lane).
 template <typename W>
-__device__ void block_select_two(const W* a, int n, int r1, int r2, int bits, unsigned* hist /*512*/,
-                                 W* shw /*4*/, W& out1, W& out2) {
-  W p1 = 0, p2 = 0, mask = 0;
-  int k1 = r1, k2 = r2;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (int hi = bits; hi > 0; hi -= 8) {
+__device__ W block_select_from(const W* a, int n, int rank, W prefix, W mask, int hi_bits, unsigned* hist,
+                               W* shw) {
+  const int lane = threadIdx.x & 31;
+  int rk = rank;
+  for (int hi = hi_bits; hi > 0; hi -= 8) {
     const int w = hi < 8 ? hi : 8, sh = hi - w;
-    const bool same = (p1 == p2);
-    for (int i = threadIdx.x; i < 512; i += blockDim.x) hist[i] = 0;
+    for (int i = threadIdx.x; i < 256; i += blockDim.x) hist[i] = 0;
     __syncthreads();
-#pragma unroll 4
     for (int i = threadIdx.x; i < n; i += blockDim.x) {
       const W v = a[i];
-      const unsigned d = (unsigned)(v >> sh) & 255u;
-      if ((v & mask) == p1) atomicAdd(&hist[d], 1u);
-      if (!same && (v & mask) == p2) atomicAdd(&hist[256 + d], 1u);
+      if ((v & mask) == prefix) atomicAdd(&hist[(unsigned)(v >> sh) & 255u], 1u);
     }
     __syncthreads();
-    if (warp < 2) {
-      const unsigned* h = hist + ((warp == 1 && !same) ? 256 : 0);
-      const int rk = (warp == 0) ? k1 : k2;
+    if (threadIdx.x < 32) {
       unsigned c[8], tot = 0;
 #pragma unroll
-      for (int t = 0; t < 8; ++t) { c[t] = h[lane * 8 + t]; tot += c[t]; }
+      for (int t = 0; t < 8; ++t) { c[t] = hist[lane * 8 + t]; tot += c[t]; }
       unsigned incl = tot;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
@@ -289,23 +277,74 @@ __device__ void block_select_two(const W* a, int n, int r1, int r2, int bits, un
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
           if (run <= (unsigned)rk && (unsigned)rk < run + c[t]) {
-            shw[warp * 2] = (W)(lane * 8 + t);
-            shw[warp * 2 + 1] = (W)run;
+            shw[0] = (W)(lane * 8 + t);
+            shw[1] = (W)run;
           }
           run += c[t];
         }
       }
     }
     __syncthreads();
-    p1 |= shw[0] << sh;
-    k1 -= (int)shw[1];
-    p2 |= shw[2] << sh;
-    k2 -= (int)shw[3];
+    prefix |= shw[0] << sh;
+    rk -= (int)shw[1];
     mask |= (W)((1u << w) - 1u) << sh;
     __syncthreads();
   }
-  out1 = p1;
-  out2 = p2;
+  return prefix;
+}
+
+// Elements of ranks r1 <= r2 among a[0..n): the first 8-bit digit of both from ONE pass over the n
+// samples; the samples in each rank's first-digit bin are then compacted into `scratch` and the
+// remaining digits run over those few only.
+template <typename W>
+__device__ void block_select_two(const W* a, W* scratch, int n, int r1, int r2, int bits, unsigned* hist,
+                                 W* shw, int* cnt, W& out1, W& out2) {
+  const int lane = threadIdx.x & 31;
+  const int sh = bits - 8;
+  for (int i = threadIdx.x; i < 256; i += blockDim.x) hist[i] = 0;
+  if (threadIdx.x < 2) cnt[threadIdx.x] = 0;
+  __syncthreads();
+  for (int i = threadIdx.x; i < n; i += blockDim.x) atomicAdd(&hist[(unsigned)(a[i] >> sh) & 255u], 1u);
+  __syncthreads();
+  if (threadIdx.x < 64) {  // warp 0: rank r1, warp 1: rank r2
+    const int wq = threadIdx.x >> 5;
+    const int rk = wq ? r2 : r1;
+    unsigned c[8], tot = 0;
+#pragma unroll
+    for (int t = 0; t < 8; ++t) { c[t] = hist[lane * 8 + t]; tot += c[t]; }
+    unsigned incl = tot;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned y = __shfl_up_sync(kFull, incl, o);
+      if (lane >= o) incl += y;
+    }
+    unsigned run = incl - tot;
+    if (run <= (unsigned)rk && (unsigned)rk < incl) {
+#pragma unroll
+      for (int t = 0; t < 8; ++t) {
+        if (run <= (unsigned)rk && (unsigned)rk < run + c[t]) {
+          shw[2 * wq] = (W)(lane * 8 + t);
+          shw[2 * wq + 1] = (W)run;
+        }
+        run += c[t];
+      }
+    }
+  }
+  __syncthreads();
+  const W d1 = shw[0], d2 = shw[2];
+  const int k1 = r1 - (int)shw[1], k2 = r2 - (int)shw[3];
+  // compaction: list 1 from the front of scratch, list 2 (if a different bin) from the back
+  for (int i = threadIdx.x; i < n; i += blockDim.x) {
+    const W v = a[i], d = (v >> sh) & 255u;
+    if (d == d1) scratch[atomicAdd(&cnt[0], 1)] = v;
+    else if (d == d2) scratch[n - 1 - atomicAdd(&cnt[1], 1)] = v;
+  }
+  __syncthreads();
+  const int n1 = cnt[0], n2 = cnt[1];
+  const W m8 = (W)255u << sh;
+  out1 = block_select_from<W>(scratch, n1, k1, d1 << sh, m8, sh, hist, shw);
+  if (d2 == d1) out2 = block_select_from<W>(scratch, n1, k2, d2 << sh, m8, sh, hist, shw);
+  else out2 = block_select_from<W>(scratch + (n - n2), n2, k2, d2 << sh, m8, sh, hist, shw);
 }
 
 constexpr int kSampleCTAs = 16;  // CTAs per row issuing the scattered sample loads (one SM cannot
@@ -316,9 +355,11 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
   extern __shared__ __align__(16) unsigned char sample_smem[];
-  W* codes = (W*)sample_smem;  // nsamp codes (last CTA only)
+  W* codes = (W*)sample_smem;           // nsamp codes (last CTA only)
+  W* scratch = codes + nsamp;           // compacted candidates of the rank selection
   __shared__ unsigned hist[512];
   __shared__ W shw[4];
+  __shared__ int sh_cnt[2];
   __shared__ int sh_last;
   const int64_t row = blockIdx.x / kSampleCTAs;
   const int part = blockIdx.x % kSampleCTAs;
@@ -382,7 +423,7 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
     return;
   }
   W lo, hi;
-  block_select_two<W>(codes, nsamp, rlo > 0 ? rlo : 0, rhi, KT<KIND>::R, hist, shw, lo, hi);
+  block_select_two<W>(codes, scratch, nsamp, rlo > 0 ? rlo : 0, rhi, KT<KIND>::R, hist, shw, sh_cnt, lo, hi);
   if (rlo <= 0) lo = 0;  // no results below the window: everything up to hi is a candidate
   if (threadIdx.x == 0) {
     st->win_lo = lo;
@@ -440,12 +481,12 @@ cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, c
   ev.record(ie++, s);
   if (nsamp > 0) {  // sample-guided window: sample, window pass (= pass 0 + filter), pass 0 over the window
     using W = std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long, unsigned>;
-    const size_t smem = (size_t)kMaxSamples * sizeof(W);
+    const size_t smem = (size_t)2 * kMaxSamples * 4;  // 8-byte keys: nsamp <= kMaxSamples / 2
     static const cudaError_t attr =
         cudaFuncSetAttribute(sample_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (attr != cudaSuccess) return attr;
     cudaError_t es = launch_pdl(sample_kernel<KIND>, dim3((unsigned)(batch * kSampleCTAs)), dim3(kSampleBlock),
-                                (size_t)nsamp * sizeof(W), s, gp, nsamp);
+                                (size_t)2 * nsamp * sizeof(W), s, gp, nsamp);
     if (es != cudaSuccess) return es;
     ev.record(ie++, s);
     cudaError_t e = launch_one<KIND, IdxT, 3, 0, HASIDX, TMA>(gp, grid, 0, 0, s);

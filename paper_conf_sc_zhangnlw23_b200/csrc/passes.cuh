@@ -194,8 +194,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
   const W kx_B = (DF == 1) ? (W)(bc << wq_) : (W)0;
   const W kx_S = (DF == 1) ? (W)((tc - bc) << wq_) : (W)0;
   const W kx_nb = (W)1 << wq_;
-  const W kx_Swin = kx_S + (emit_all ? kx_nb : (W)0);
-  const W kx_nbS = store ? kx_nb : (W)0;
+  const W kx_flag = kx_S + ((emit_all || store) ? kx_nb : (W)0);  // fast-path flag threshold on y
   // shared-window address of this lane's histogram copy (c.hist is the dynamic smem base)
   const unsigned hbase = (unsigned)__cvta_generic_to_shared(c.hist) + ((HC > 1) ? (unsigned)(lane % HC) * 4u : 0u);
   const U xmask = sel_min ? (U)0 : (U)~(U)0;
@@ -210,6 +209,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
   };
   // Filter classification of digit q-1 (Alg1 L15-22): win = result, cand = candidate for pass q.
   const W wlo = (W)c.lo, wspan = (W)c.span1;
+  const W whi = (W)(wlo + wspan - 1);  // DF == 3: window [lo, hi]
   auto classify = [&](U code, IdxT idx, bool valid, bool& win, bool& cand) {
     bool lt, eq;
     if constexpr (DF == 3) {  // sample-guided window
@@ -281,16 +281,16 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
       using FlagT = std::conditional_t<(kUnroll * VEC > 32), unsigned long long, unsigned>;
       FlagT fl = 0;  // elements that must leave through the queues (results / stored candidates)
       if constexpr (DF == 3) {
-        // window pass: results below the window -> output, window members -> candidate buffer;
-        // pure filter (no histogram): a miss is repaired by re-running the paper's pass 1
+        // window pass: results below the window -> output, window members -> candidate buffer and
+        // (slow path) the pass-1 histogram of the window members; a miss re-runs the paper's pass 1
 #pragma unroll
         for (int u = 0; u < kUnroll; ++u) {
           const bool valid = FULL || (vb + (int64_t)u * vs < vlim);
 #pragma unroll
           for (int e = 0; e < VEC; ++e) {
             const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
-            const bool sel = ((W)code < wlo) || ((W)((W)code - wlo) < wspan);
-            if (valid && sel) fl |= (FlagT)1 << (u * VEC + e);
+            // result (code < lo) or window member (lo <= code <= hi): together simply code <= hi
+            if (valid && (W)code <= whi) fl |= (FlagT)1 << (u * VEC + e);
           }
         }
       } else if constexpr (DF == 1 && DH == 1) {
@@ -303,12 +303,10 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
           for (int e = 0; e < VEC; ++e) {
             const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
             const W y = ((W)code >> shh) - kx_B;
-            const W x = y - kx_S;
-            const bool win = y < kx_Swin;
-            const bool cst = x < kx_nbS;
-            const unsigned d = (unsigned)min(x, (W)kDummyBin);
+            const unsigned d = (unsigned)min((W)(y - kx_S), (W)kDummyBin);
             shared_inc(hbase + (valid ? d : (unsigned)kDummyBin) * (HC * 4u));
-            if (valid && (win || cst)) fl |= (FlagT)1 << (u * VEC + e);
+            // result (y < S) or stored candidate / emit-all member (S <= y < S + nb): one compare
+            if (valid && y < kx_flag) fl |= (FlagT)1 << (u * VEC + e);
           }
         }
       } else {
@@ -361,9 +359,10 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
         bool w, cd;
         classify(code, idx, has, w, cd);
         if constexpr (DF == 3) {
-          if (cd) {
+          if (cd) {  // window member: extremes + the pass-1 digit histogram of the window buffer
             wlo_seen = ((W)code < wlo_seen) ? (W)code : wlo_seen;
             whi_seen = ((W)code > whi_seen) ? (W)code : whi_seen;
+            shared_inc(hbase + 4u * (unsigned)((W)code >> shh));
           }
         }
         push_out(w, code, idx);
@@ -482,6 +481,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
           if (cand) {
             wlo_seen = ((W)code < wlo_seen) ? (W)code : wlo_seen;
             whi_seen = ((W)code > whi_seen) ? (W)code : whi_seen;
+            shared_inc(hbase + 4u * (unsigned)((W)code >> shh));
           }
         }
         push_out(win, code, idx);
