@@ -2,6 +2,7 @@
 # Round deliverable run: full bench (default c3 + extras + cpu baseline), reference arm, ncu launch list
 # and --set full captures of the dominant kernels, gpu tests.
 mkdir -p gpurun_out
+rm -f gpurun_out/bench_*.json gpurun_out/*.ncu-rep gpurun_out/launches_*.csv
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > gpurun_out/smi.txt
 timeout 900 python -m pytest tests -m gpu -q --timeout 300 2>&1 | tail -5 > gpurun_out/pytest_gpu.log
 python bench.py > gpurun_out/bench_full.json 2> gpurun_out/bench_full.err
@@ -13,6 +14,7 @@ timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__byte
 timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -c 40 --csv --log-file gpurun_out/launches_c4.csv python tools/prof_select.py --config c4 --reps 3 > /dev/null 2>&1
 timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -c 60 --csv --log-file gpurun_out/launches_c2.csv python tools/prof_select.py --config c2 --reps 3 > /dev/null 2>&1
 # one full capture of the dominant kernel per path (window pass; paper pass 1 and 2)
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:pass_kernel -s 9 -c 1 -o gpurun_out/full_c3_window python tools/prof_select.py --config c3 --reps 2 > gpurun_out/ncu_w.log 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:pass_kernel -s 8 -c 1 -o gpurun_out/full_c3_window python tools/prof_select.py --config c3 --reps 2 > gpurun_out/ncu_w.log 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:cluster_kernel -s 1 -c 1 -o gpurun_out/full_c4_tail python tools/prof_select.py --config c4 --reps 2 > gpurun_out/ncu_t.log 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:pass_kernel -s 7 -c 2 -o gpurun_out/full_c3_paper python tools/prof_select.py --config c3 --reps 2 --window -1 > gpurun_out/ncu_p.log 2>&1
 ls -la gpurun_out | tail -30
