@@ -177,6 +177,8 @@ def main():
     ap.add_argument("--ref-budget", type=float, default=20.0)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--engine", type=int, default=0, help="0 auto, 1 grid, 2 cluster (ablations)")
+    ap.add_argument("--dtype", default="f32", choices=["f32", "f16", "bf16", "f64", "u32"],
+                    help="key type (f32: the paper's; others: the config's f32 keys converted)")
     ap.add_argument("--window", type=int, default=0, help="sample-guided window: 0 auto, 1 on, -1 off (ablation)")
     ap.add_argument("--tma", type=int, default=0, help="bulk-copy streaming: 0 auto, 1 on, -1 off (ablation)")
     ap.add_argument("--dist-backend", default="nccl", help="nccl (default); gloo only to self-test the "
@@ -229,13 +231,16 @@ def main():
         total_units = world * batch * n
         split = world > 1
     k = c["k"]
-    xd = torch.from_numpy(xh).to(dev)
+    xt = keys_as(torch.from_numpy(xh), args.dtype)
+    kdt = xt.dtype
+    esz = xt.element_size()
+    xd = xt.to(dev)
     sel_opts = dict(engine=args.engine, window=args.window, tma=args.tma)
-    ws = torch.empty(max(1, at.describe(torch.float32, batch, n, k, **sel_opts)["workspace_bytes"]),
+    ws = torch.empty(max(1, at.describe(kdt, batch, n, k, **sel_opts)["workspace_bytes"]),
                      dtype=torch.uint8, device=dev)
-    ov = torch.empty((batch, k), dtype=torch.float32, device=dev)
+    ov = torch.empty((batch, k), dtype=kdt, device=dev)
     oi = torch.empty((batch, k), dtype=torch.int64, device=dev)
-    plan = at.describe(torch.float32, batch, n, k, **sel_opts)
+    plan = at.describe(kdt, batch, n, k, **sel_opts)
     n_launch = plan["launches"]
     stream = torch.cuda.current_stream(dev)
     ev_sets = []
@@ -296,8 +301,8 @@ def main():
     per /= args.steps
     select_ms = float(per.sum())
     dom = int(np.argmax(per))
-    in_bytes = batch * n * 4
-    out_bytes = batch * k * (4 + 8)
+    in_bytes = batch * n * esz
+    out_bytes = batch * k * (esz + 8)
     # algorithmic bytes of the dominant kernel: passes that read the input read N*4 bytes once
     # (grid engine: launch 0 and 1 read L; cluster engine: its single launch reads the rows)
     names, reads_L = launch_names(plan)
@@ -322,7 +327,7 @@ def main():
             "metric": "top-K elements/s and achieved HBM GB/s vs B200 peak (N=2^30,K=2^20; b=100)",
             "value": value, "unit": "elements/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": ms, "higher_is_better": True, "scaling": scaling, "vs_baseline": None,
-            "dtype": "f32", "data": "synthetic",
+            "dtype": args.dtype, "data": "synthetic",
             "config": {"workload": cfg, "batch": c["batch"], "n": n, "k": k, "dist": c["dist"], "select": "min",
                        "per_gpu_rows": batch, "split_row": split,
                        "l2": "input (%.2f GB) larger than L2 (126 MB): no flush needed" % (in_bytes / 1e9)
@@ -338,8 +343,8 @@ def main():
         }
     # ---------------- e2e through the C ABI with HOST buffers (pinned), N GPUs, same metric
     if True:
-        xpin = torch.from_numpy(xh).pin_memory()
-        ovh = torch.empty((batch, k), dtype=torch.float32).pin_memory()
+        xpin = xt.pin_memory()
+        ovh = torch.empty((batch, k), dtype=kdt).pin_memory()
         oih = torch.empty((batch, k), dtype=torch.int64).pin_memory()
         at.select_host(xpin, k, out=(ovh, oih))
         if world > 1:
@@ -361,9 +366,10 @@ def main():
     if rank == 0:
         # oracle-free sanity of the timed output: K distinct indices, values = keys[idx]
         ii = i_chk.reshape(-1)[: min(k, 4096)].cpu().numpy()
-        vv = v_chk.reshape(-1)[: min(k, 4096)].cpu().numpy()
         if not split:
-            assert np.array_equal(xh.reshape(-1)[ii].view(np.uint32), vv.view(np.uint32)), "value/index mismatch"
+            xb = xt.reshape(-1).view({1: torch.uint8, 2: torch.int16, 4: torch.int32, 8: torch.int64}[esz])
+            vb = v_chk.reshape(-1)[: min(k, 4096)].view(xb.dtype).cpu()
+            assert torch.equal(xb[torch.from_numpy(ii)], vb), "value/index mismatch"
         if not args.no_cpu:
             result["cpu_baseline"] = cpu_sample_run(cfg, args.cpu_budget)
         if world == 1 and not args.no_extras and cfg == "c3":
@@ -376,6 +382,21 @@ def main():
         dist.destroy_process_group()
 
 
+def keys_as(xt, dtype):
+    """The config's f32 keys as another key type (f16/bf16/f64 by value conversion, u32 by the
+    order-preserving bit pattern of the positive f32 values)."""
+    import torch
+    if dtype == "f32":
+        return xt
+    if dtype == "f16":
+        return xt.half()
+    if dtype == "bf16":
+        return xt.bfloat16()
+    if dtype == "f64":
+        return xt.double()
+    return xt.view(torch.int32).view(torch.uint32)
+
+
 def launch_names(plan):
     """Names of a select's launches in order, and whether each streams the input row L once (its
     algorithmic bytes are then N*4; SURVEY §8(d) per-element figure x elements per launch)."""
@@ -384,7 +405,13 @@ def launch_names(plan):
     if plan["engine"] == 3:
         return ["trivial_copy"], [True]
     P = plan["passes"]
-    window = plan["launches"] == P + 3
+    L = plan["launches"]
+    if L not in (P + 1, P + 3):  # window pass + tail_q grid passes + one cluster-engine tail launch
+        tq = L - 3
+        names = ["sample_kernel", "window_pass (DF=3)"] + [f"pass_kernel q={q} [window buffer]" for q in range(tq)]
+        names.append("cluster_kernel (tail)")
+        return names, [False, True] + [False] * (tq + 1)
+    window = L == P + 3
     names, reads = [], []
     if window:
         names += ["sample_kernel", "window_pass (DF=3)"]

@@ -25,6 +25,8 @@ int bits_needed(uint64_t v) {  // number of bits to represent v (0 for v == 0)
   return b;
 }
 
+}  // namespace
+
 int num_sms() {
   static thread_local int dev_cached = -1, sms_cached = 148;
   int dev = 0;
@@ -36,7 +38,6 @@ int num_sms() {
   }
   return sms_cached;
 }
-}  // namespace
 
 int key_bits(int kind) {
   switch (kind) {
@@ -108,6 +109,8 @@ static int auto_cluster_size(const SelectArgs& a) {
   return cs;
 }
 
+constexpr double kTailPerCTA = 4096.0;  // expected window entries per cluster-tail CTA
+
 static void choose_launch(const SelectArgs& a, Plan& p) {
   if (p.engine == 3) return;
   p.engine = a.engine > 0 ? a.engine : auto_engine(a);
@@ -121,10 +124,15 @@ static void choose_launch(const SelectArgs& a, Plan& p) {
     const double f = (double)a.k / (double)a.len, r = f * p.nsamp;
     const double rhi = r + 4.0 * std::sqrt(r * (1.0 - f)) + 9.0;  // sample_kernel's margin
     const double expect = rhi / p.nsamp * (double)a.len;
-    if (expect <= (double)(1 << 20) && a.engine == 0) {
+    // small windows: one cluster-engine launch runs every pass after the window pass. (Measured: a
+    // tail CTA needs ~25 us per pass at ~20K window entries, where the 444-CTA grid passes are
+    // faster, so the tail is kept for windows of <= 4K entries per CTA of a cluster of <= 16;
+    // tail_q > 0 — grid passes first, then the tail — is supported but off.)
+    if (a.engine == 0 && expect <= 16.0 * kTailPerCTA) {
       p.tail = 1;
+      p.tail_q = 0;
       int cs = 1;
-      while (cs < 16 && cs * 16384.0 < expect) cs <<= 1;
+      while (cs < 16 && cs * kTailPerCTA < expect) cs <<= 1;
       p.csize = a.cluster_size > 0 ? a.cluster_size : cs;
     }
   }
@@ -134,7 +142,7 @@ static void choose_launch(const SelectArgs& a, Plan& p) {
       (a.tma > 0 || (a.batch * 2 <= num_sms() && a.len >= (int64_t(1) << 22))))
     p.tma = 1;
   if (a.ctas_per_row > 0) {
-    p.cpr = a.ctas_per_row;
+    p.cpr = p.cpr_buf = a.ctas_per_row;
     return;
   }
   const int64_t target = (int64_t)num_sms() * (p.tma ? 1 : grid_blocks_per_sm(a, p.idx64));
@@ -143,6 +151,10 @@ static void choose_launch(const SelectArgs& a, Plan& p) {
   // whole waves: batch x cpr <= target CTAs (a partial second wave costs more than idle slots)
   int64_t c = std::max<int64_t>(1, target / a.batch);
   p.cpr = (int)std::max<int64_t>(1, std::min<int64_t>(c, maxc));
+  // After a bulk-copy window pass the next passes read the (small) window buffer: they run the
+  // register-load kernel, whose 3 CTAs/SM hide the queue and load latencies (measured 2-3x faster).
+  const int64_t cb = std::max<int64_t>(1, (int64_t)num_sms() * grid_blocks_per_sm(a, p.idx64) / a.batch);
+  p.cpr_buf = p.tma ? (int)std::max<int64_t>(1, std::min<int64_t>(cb, maxc)) : p.cpr;
 }
 
 static bool valid_kind(int dt) { return dt >= AIRTOPK_F32 && dt <= AIRTOPK_U32; }
@@ -355,7 +367,7 @@ airtopk_status airtopk_describe(airtopk_dtype dtype, int64_t batch, int64_t len,
   std::memset(out, 0, sizeof(*out));
   out->engine = p.engine;
   out->passes = p.P;
-  out->launches = p.engine == 3 ? 1 : (p.engine == 2 ? 1 : (p.tail ? 3 : p.P + 1 + (p.nsamp > 0 ? 2 : 0)));
+  out->launches = p.engine == 3 ? 1 : (p.engine == 2 ? 1 : (p.tail ? 3 + p.tail_q : p.P + 1 + (p.nsamp > 0 ? 2 : 0)));
   out->ctas_per_row = p.engine == 1 ? p.cpr : 0;
   out->cluster_size = (p.engine == 2 || p.tail) ? p.csize : 0;
   out->index_bits = p.IB;

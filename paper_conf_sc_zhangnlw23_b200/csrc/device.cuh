@@ -150,6 +150,15 @@ __device__ __forceinline__ unsigned long long warp_alloc(bool pred, unsigned lon
   return base + __popc(mask & lanemask_lt());
 }
 
+// "Last thread block" ticket: a device-scope acq_rel fetch-add. The release publishes the
+// calling CTA's prior global writes (ordered before it by the __syncthreads that precedes the call);
+// the acquire lets the last arriving CTA read everyone's. Cheaper than __threadfence (fence.sc.gpu).
+__device__ __forceinline__ unsigned ticket_arrive(unsigned* t) {
+  unsigned old;
+  asm volatile("atom.add.acq_rel.gpu.u32 %0, [%1], 1;" : "=r"(old) : "l"(t) : "memory");
+  return old;
+}
+
 // Programmatic dependent launch (PDL): wait for the previous kernel in the stream (its writes are
 // then visible), and let the next kernel's CTAs be scheduled as ours retire. No-ops without PDL.
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }

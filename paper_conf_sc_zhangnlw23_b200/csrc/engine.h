@@ -37,15 +37,18 @@ struct Plan {
   int64_t cap_rule;  // buffer iff C <= cap_rule  (== C * alpha < N)
   int64_t cap_alloc; // entries allocated per candidate buffer
   int cpr;           // CTAs per row (grid engine)
+  int cpr_buf;       // CTAs per row of the register-load passes after a bulk-copy window pass
   int csize;         // CTAs per cluster (cluster engine)
   int max_clusters;  // cluster engine: clusters the workspace has candidate buffers for
   int nsamp;         // grid engine: samples per row for the sample-guided window (0 = off)
   int tail;          // grid engine: finish after the window pass with one cluster-engine launch
+  int tail_q;        // ... after the grid passes q < tail_q (0: right after the window pass)
   int tma;           // grid engine: stream rows through bulk-copy (TMA) shared rings, 1 CTA/SM
   size_t off_state, off_hist, off_bcode, off_bidx, off_samp, bytes;
 };
 
 int key_bits(int kind);
+int num_sms();  // SMs of the current device (cached per thread)
 int key_bytes(int kind);
 Plan make_plan(const SelectArgs& a);
 cudaError_t run_grid(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);

@@ -44,7 +44,8 @@ struct ClusterParams {
   int64_t cap_rule, cap_alloc;
   int nclusters;
   int tail;      // 1: continue rows after the grid engine's window pass
-  int64_t* timing;  // optional: per CTA [globaltimer at start, at end, rows done, passes run]
+  int tail_q;    // tail mode: the grid engine ran passes q < tail_q after the window pass
+  int64_t* timing;  // optional: per CTA [globaltimer at start, at end, rows done, passes run, end of passes 1-4]
 };
 
 struct ClusterShared {
@@ -59,7 +60,9 @@ struct ClusterShared {
 // costs more than the same-bin serialisation they avoid.
 template <int KIND, typename IdxT, int DF, int DH, bool HASIDX>
 __device__ __forceinline__ unsigned long long cluster_pass(PassCtx<typename KT<KIND>::U, IdxT>& c) {
-  return run_pass<KIND, IdxT, DF, DH, HASIDX, kCBlock, 1>(c);
+  // 8 buffer entries per thread per iteration: the few CTAs of a cluster need deep memory-level
+  // parallelism to stream a candidate buffer from L2
+  return run_pass<KIND, IdxT, DF, DH, HASIDX, kCBlock, 1, false, 8>(c);
 }
 
 template <int KIND, typename IdxT, bool HASIDX>
@@ -92,16 +95,20 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
     unsigned long long K = kk, C = N, Cp = N, tcode = 0, tidx = 0;
     int stop1 = 0, src1 = 0;  // src1: 0 = the input row L, s + 1 = candidate buffer slot s
     int q0 = 0;
-    if (p.tail && st->win_state == 1) {
-      // the window held the K-th key and the window pass already scanned pass 1 over the window
-      // buffer: continue from its state
+    const int ws = p.tail ? st->win_state : 0;
+    if (p.tail && (ws == 1 || p.tail_q > 0)) {
+      // continue the row from its state: after the window pass (which scanned pass 1 over the window
+      // buffer) or after the grid passes q < tail_q
       K = st->K;
       C = st->C;
       Cp = st->Cp;
       src1 = st->src1;
       tcode = st->tcode;
+      tidx = st->tidx;
       stop1 = st->stop1;
       q0 = st->npass;
+    }
+    if (ws == 1) {
       // Every window member lies in [wmin, wmax]: while all key bits above digit q agree between the
       // two (so no result of an earlier digit is pending), pass q's histogram is a single bin (j = that
       // digit, K and C unchanged) and the pass is skipped — the paper's adaptivity applied to the
@@ -170,6 +177,11 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
         default: cluster_pass<KIND, IdxT, 2, 0, HASIDX>(c); break;
       }
       ++n_passes;
+      if (p.timing && tid == 0 && n_passes <= 4) {
+        unsigned long long tp;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tp));
+        p.timing[(int64_t)blockIdx.x * 8 + 3 + n_passes] = (int64_t)tp;
+      }
       if (!hist_on) break;  // emit-all pass: the row is complete
 
       // ---- histogram merge + scan (replaces the last-block scan) ----
@@ -249,7 +261,7 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
   if (p.timing && tid == 0) {
     unsigned long long t_end;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
-    int64_t* t = p.timing + (int64_t)blockIdx.x * 4;
+    int64_t* t = p.timing + (int64_t)blockIdx.x * 8;
     t[0] = (int64_t)t_start; t[1] = (int64_t)t_end; t[2] = n_rows; t[3] = n_passes;
   }
 }
@@ -289,6 +301,7 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   p.cap_rule = pl.cap_rule;
   p.cap_alloc = pl.cap_alloc;
   p.tail = tail;
+  p.tail_q = pl.tail_q;
   p.timing = a.trace;  // cluster engine: the trace buffer receives per-CTA timing instead
 
   cudaLaunchConfig_t cfg = {};

@@ -57,8 +57,10 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t
   gp.cap_rule = pl.cap_rule;
   gp.cap_alloc = pl.cap_alloc;
   gp.cpr = pl.cpr;
+  gp.cpr_buf = pl.cpr_buf;
   gp.trace = a.trace;
   gp.samp = base + pl.off_samp;
+  gp.nsms = num_sms();
   switch (a.kind) {
     case K_F32: return launch_grid_kind<K_F32>(a, pl, gp, ws, s);
     case K_F16: return launch_grid_kind<K_F16>(a, pl, gp, ws, s);

@@ -60,8 +60,10 @@ struct GridParams {
   void* bidx;
   int64_t cap_rule, cap_alloc;
   int cpr;
+  int cpr_buf;  // passes q >= 1 after a bulk-copy window pass (they read the window buffer)
   int64_t* trace;
   void* samp;  // sample-guided window: [batch][nsamp] sampled codes
+  int nsms;    // SMs of the device
 };
 
 constexpr int kBlock = 512;
@@ -178,12 +180,10 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
     for (int h = 0; h < HC; ++h) v += sh_hist[i * HC + h];
     if (v) atomicAdd(&gh[i], (CountT)v);
   }
-  __threadfence();
-  __syncthreads();
-  if (tid == 0) sh_last = (atomicAdd(&st->ticket, 1u) == (unsigned)(p.cpr - 1));
+  __syncthreads();  // the CTA's histogram merge / queue flushes precede thread 0's release
+  if (tid == 0) sh_last = (ticket_arrive(&st->ticket) == (unsigned)(p.cpr - 1));
   __syncthreads();
   if (!sh_last) return;
-  __threadfence();
 
   const unsigned long long kk = (unsigned long long)p.k;
   unsigned long long Kin = (FILTER || redo_buf) ? st->K : kk;
@@ -246,20 +246,20 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
 constexpr int kSampleBlock = 1024;
 constexpr int kMaxSamples = 16384;
 
-// Rank select among a[0..n) in shared memory with 8-bit MSD digits, below a fixed prefix (bits above
-// `hi_bits` equal `prefix` under `mask`). The 256-bin scan is done by warp 0 (8 bins per lane).
+// Radix rank select over a[0..n) in shared memory, 8-bit MSD digits for bits [lo_bits, hi_bits):
+// elements outside (v & mask) == prefix are ignored; prefix / mask / rank are updated in place (every
+// thread holds the same values). The 256-bin scan is done by warp 0 (8 bins per lane + shuffles).
 template <typename W>
-__device__ W block_select_from(const W* a, int n, int rank, W prefix, W mask, int hi_bits, unsigned* hist,
-                               W* shw) {
+__device__ void select_digits(const W* a, int n, int& rank, W& prefix, W& mask, int hi_bits, int lo_bits,
+                              unsigned* hist /* 256 */, W* shw) {
   const int lane = threadIdx.x & 31;
-  int rk = rank;
-  for (int hi = hi_bits; hi > 0; hi -= 8) {
-    const int w = hi < 8 ? hi : 8, sh = hi - w;
+  for (int hi = hi_bits; hi > lo_bits; hi -= 8) {
+    const int w = (hi - lo_bits) < 8 ? (hi - lo_bits) : 8, sh = hi - w;
     for (int i = threadIdx.x; i < 256; i += blockDim.x) hist[i] = 0;
     __syncthreads();
     for (int i = threadIdx.x; i < n; i += blockDim.x) {
       const W v = a[i];
-      if ((v & mask) == prefix) atomicAdd(&hist[(unsigned)(v >> sh) & 255u], 1u);
+      if ((v & mask) == prefix) atomicAdd(&hist[(unsigned)(v >> sh) & ((1u << w) - 1u)], 1u);
     }
     __syncthreads();
     if (threadIdx.x < 32) {
@@ -273,10 +273,10 @@ __device__ W block_select_from(const W* a, int n, int rank, W prefix, W mask, in
         if (lane >= o) incl += y;
       }
       unsigned run = incl - tot;
-      if (run <= (unsigned)rk && (unsigned)rk < incl) {
+      if (run <= (unsigned)rank && (unsigned)rank < incl) {
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
-          if (run <= (unsigned)rk && (unsigned)rk < run + c[t]) {
+          if (run <= (unsigned)rank && (unsigned)rank < run + c[t]) {
             shw[0] = (W)(lane * 8 + t);
             shw[1] = (W)run;
           }
@@ -286,85 +286,170 @@ __device__ W block_select_from(const W* a, int n, int rank, W prefix, W mask, in
     }
     __syncthreads();
     prefix |= shw[0] << sh;
-    rk -= (int)shw[1];
+    rank -= (int)shw[1];
     mask |= (W)((1u << w) - 1u) << sh;
     __syncthreads();
   }
-  return prefix;
 }
 
-// Elements of ranks r1 <= r2 among a[0..n): the first 8-bit digit of both from ONE pass over the n
-// samples; the samples in each rank's first-digit bin are then compacted into `scratch` and the
-// remaining digits run over those few only.
-template <typename W>
-__device__ void block_select_two(const W* a, W* scratch, int n, int r1, int r2, int bits, unsigned* hist,
-                                 W* shw, int* cnt, W& out1, W& out2) {
-  const int lane = threadIdx.x & 31;
-  const int sh = bits - 8;
-  for (int i = threadIdx.x; i < 256; i += blockDim.x) hist[i] = 0;
+// Sample order statistics at ranks rlo (skipped when < 0) and rhi in one sweep over the samples
+// held in registers (v[t] = sample t * blockDim + tid, valid for t < tv): one 11-bit digit below the
+// common prefix (bits [hb-11, hb)), block-wide scan of 2048 bins (2 per thread), compaction of the
+// one or two chosen bins into `scratch`, then the exact rank inside each bin by counting (bins of
+// <= kBrute samples) or, for concentrated samples, 8-bit digits over the bin (select_digits).
+// Written for a short critical path: no loop carries a shared-memory load-atomic chain.
+constexpr int kBrute = 128;
+
+template <typename W, int PER>
+__device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo, int rhi, W pmin, int hb,
+                                 unsigned* hist /* 2048 */, unsigned* wsum /* 32 */, W* shw, int* cnt,
+                                 W& lo, W& hi) {
+  constexpr int WB = 8 * (int)sizeof(W);
+  if (hb <= 0) {  // all samples equal
+    lo = hi = pmin;
+    return;
+  }
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int w = hb < 11 ? hb : 11, sh = hb - w;
+  const unsigned dmask = (1u << w) - 1u;
+  const W mask = (hb >= WB) ? (W)0 : (W)(~(W)0 << hb);
+  const W prefix = pmin & mask;
+  for (int i = threadIdx.x; i < 2048; i += blockDim.x) hist[i] = 0;
   if (threadIdx.x < 2) cnt[threadIdx.x] = 0;
   __syncthreads();
-  for (int i = threadIdx.x; i < n; i += blockDim.x) atomicAdd(&hist[(unsigned)(a[i] >> sh) & 255u], 1u);
+#pragma unroll
+  for (int t = 0; t < PER; ++t)
+    if (t < tv) atomicAdd(&hist[(unsigned)(v[t] >> sh) & dmask], 1u);
   __syncthreads();
-  if (threadIdx.x < 64) {  // warp 0: rank r1, warp 1: rank r2
-    const int wq = threadIdx.x >> 5;
-    const int rk = wq ? r2 : r1;
-    unsigned c[8], tot = 0;
+  // block scan: thread t owns bins 2t, 2t+1 (1024 threads)
+  const unsigned c0 = hist[2 * threadIdx.x], c1 = hist[2 * threadIdx.x + 1], tot = c0 + c1;
+  unsigned incl = tot;
 #pragma unroll
-    for (int t = 0; t < 8; ++t) { c[t] = hist[lane * 8 + t]; tot += c[t]; }
-    unsigned incl = tot;
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned y = __shfl_up_sync(kFull, incl, o);
+    if (lane >= o) incl += y;
+  }
+  if (lane == 31) wsum[warp] = incl;
+  __syncthreads();
+  unsigned wi = wsum[lane];
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const unsigned y = __shfl_up_sync(kFull, incl, o);
-      if (lane >= o) incl += y;
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned y = __shfl_up_sync(kFull, wi, o);
+    if (lane >= o) wi += y;
+  }
+  const unsigned wex = warp ? __shfl_sync(kFull, wi, warp - 1) : 0u;
+  const unsigned s0 = wex + incl - tot, s1 = s0 + c0;
+  // shw[0..1]: chosen bin of rank lo / hi, shw[2..3]: samples before it (one writer each)
+  if (rlo >= 0) {
+    if (s0 <= (unsigned)rlo && (unsigned)rlo < s1) { shw[0] = 2 * threadIdx.x; shw[2] = s0; }
+    if (s1 <= (unsigned)rlo && (unsigned)rlo < s1 + c1) { shw[0] = 2 * threadIdx.x + 1; shw[2] = s1; }
+  }
+  if (s0 <= (unsigned)rhi && (unsigned)rhi < s1) { shw[1] = 2 * threadIdx.x; shw[3] = s0; }
+  if (s1 <= (unsigned)rhi && (unsigned)rhi < s1 + c1) { shw[1] = 2 * threadIdx.x + 1; shw[3] = s1; }
+  __syncthreads();
+  const unsigned blo = (rlo >= 0) ? (unsigned)shw[0] : 0xffffffffu, bhi = (unsigned)shw[1];
+  const int rk_lo = rlo - (int)shw[2], rk_hi = rhi - (int)shw[3];
+  const int m_lo = (rlo >= 0) ? (int)hist[blo] : 0, m_hi = (int)hist[bhi];
+  const W plo = prefix | ((W)blo << sh), phi = prefix | ((W)bhi << sh);
+  if (sh == 0) {
+    lo = plo;
+    hi = phi;
+    return;
+  }
+  // compaction from registers: per-thread counts, one warp scan, one shared atomic per warp and bin
+  const bool same = (blo == bhi);
+  W* reg_lo = scratch;
+  W* reg_hi = same ? scratch : scratch + m_lo;
+  unsigned cl = 0, ch = 0;
+#pragma unroll
+  for (int t = 0; t < PER; ++t) {
+    const unsigned d = (unsigned)(v[t] >> sh) & dmask;
+    cl += (t < tv) && d == blo;
+    ch += (t < tv) && !same && d == bhi;
+  }
+  unsigned pk = cl | (ch << 16), pki = pk;  // <= 16 per thread, <= 512 per warp: 16-bit fields
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned y = __shfl_up_sync(kFull, pki, o);
+    if (lane >= o) pki += y;
+  }
+  unsigned base = 0;
+  if (lane == 31 && pki) {
+    const unsigned bl = (pki & 0xffffu) ? (unsigned)atomicAdd(&cnt[0], (int)(pki & 0xffffu)) : 0u;
+    const unsigned bh = (pki >> 16) ? (unsigned)atomicAdd(&cnt[1], (int)(pki >> 16)) : 0u;
+    base = bl | (bh << 16);
+  }
+  base = __shfl_sync(kFull, base, 31);
+  if (pk) {
+    unsigned ol = (base & 0xffffu) + ((pki - pk) & 0xffffu), oh = (base >> 16) + ((pki - pk) >> 16);
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+      const unsigned d = (unsigned)(v[t] >> sh) & dmask;
+      if (t < tv && d == blo) reg_lo[ol++] = v[t];
+      else if (t < tv && !same && d == bhi) reg_hi[oh++] = v[t];
     }
-    unsigned run = incl - tot;
-    if (run <= (unsigned)rk && (unsigned)rk < incl) {
-#pragma unroll
-      for (int t = 0; t < 8; ++t) {
-        if (run <= (unsigned)rk && (unsigned)rk < run + c[t]) {
-          shw[2 * wq] = (W)(lane * 8 + t);
-          shw[2 * wq + 1] = (W)run;
+  }
+  __syncthreads();
+  // exact rank inside a bin
+  const W sub = (W)dmask << sh;
+  W res[2] = {plo, phi};
+  for (int q = (rlo >= 0 ? 0 : 1); q < 2; ++q) {
+    const W* reg = q ? reg_hi : reg_lo;
+    const int m = q ? m_hi : m_lo;
+    int rk = q ? rk_hi : rk_lo;
+    if (m <= kBrute) {
+      if ((int)threadIdx.x < m) {
+        const W x = reg[threadIdx.x];
+        int less = 0, eq = 0;
+        for (int j = 0; j < m; ++j) {
+          const W u = reg[j];
+          less += u < x;
+          eq += u == x;
         }
-        run += c[t];
+        if (less <= rk && rk < less + eq) shw[4 + q] = x;
       }
+      __syncthreads();
+      res[q] = shw[4 + q];
+    } else {
+      W pre = res[q], msk = mask | sub;
+      select_digits<W>(reg, m, rk, pre, msk, sh, 0, hist, shw + 6);
+      res[q] = pre;
     }
   }
-  __syncthreads();
-  const W d1 = shw[0], d2 = shw[2];
-  const int k1 = r1 - (int)shw[1], k2 = r2 - (int)shw[3];
-  // compaction: list 1 from the front of scratch, list 2 (if a different bin) from the back
-  for (int i = threadIdx.x; i < n; i += blockDim.x) {
-    const W v = a[i], d = (v >> sh) & 255u;
-    if (d == d1) scratch[atomicAdd(&cnt[0], 1)] = v;
-    else if (d == d2) scratch[n - 1 - atomicAdd(&cnt[1], 1)] = v;
-  }
-  __syncthreads();
-  const int n1 = cnt[0], n2 = cnt[1];
-  const W m8 = (W)255u << sh;
-  out1 = block_select_from<W>(scratch, n1, k1, d1 << sh, m8, sh, hist, shw);
-  if (d2 == d1) out2 = block_select_from<W>(scratch, n1, k2, d2 << sh, m8, sh, hist, shw);
-  else out2 = block_select_from<W>(scratch + (n - n2), n2, k2, d2 << sh, m8, sh, hist, shw);
+  lo = res[0];
+  hi = res[1];
 }
 
-constexpr int kSampleCTAs = 16;  // CTAs per row issuing the scattered sample loads (one SM cannot
+constexpr int kSampleCTAs = 16;  // max CTAs per row issuing the scattered sample loads (one SM cannot
                                  // keep 16K independent DRAM loads in flight)
 
 template <int KIND>
-__global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p, int nsamp) {
+__global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p, int nsamp, int cps) {
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
   extern __shared__ __align__(16) unsigned char sample_smem[];
-  W* codes = (W*)sample_smem;           // nsamp codes (last CTA only)
-  W* scratch = codes + nsamp;           // compacted candidates of the rank selection
-  __shared__ unsigned hist[512];
-  __shared__ W shw[4];
-  __shared__ int sh_cnt[2];
+  W* scratch = (W*)sample_smem;  // nsamp entries: compacted bins of the rank selection (last CTA)
+  __shared__ unsigned hist[2048];
+  __shared__ unsigned wsum[32];
+  __shared__ W shw[8];
+  __shared__ int sh_cnt[4];
+  __shared__ W sh_red[64];
   __shared__ int sh_last;
-  const int64_t row = blockIdx.x / kSampleCTAs;
-  const int part = blockIdx.x % kSampleCTAs;
+  const int64_t row = blockIdx.x / cps;
+  const int part = blockIdx.x % cps;
   RowState* st = p.st + row;
+  // debug timing (trace slot 15 of the row): t0 start, t1 after pdl_wait, t2 ticket won, t3 codes in
+  // smem, t4 selection done
+  auto stamp = [&](int f) {
+    if (p.trace && threadIdx.x == 0) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      p.trace[((size_t)row * kTraceMaxPasses + (kTraceMaxPasses - 1)) * kTraceFields + f] = (int64_t)t;
+    }
+  };
+  if (part == 0) stamp(0);
   pdl_wait();
+  if (part == 0) stamp(1);
   pdl_trigger();
   const U* rowp = (const U*)p.keys + row * p.len;
   W* samp = (W*)p.samp + row * (int64_t)nsamp;
@@ -376,40 +461,62 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
   constexpr int kRun = 32;
   const int nruns = nsamp / kRun;
   const int64_t stride = p.len / nruns;
-  // phase 1: this CTA's runs part, part + 16, ... (all loads in flight at once)
+  // phase 1: this CTA's runs part, part + cps, ... (all loads in flight at once)
   {
-    constexpr int PER = kMaxSamples / (kSampleBlock * kSampleCTAs);
+    constexpr int PER = kMaxSamples / kSampleBlock;
+    const int runs_here = (nruns - part + cps - 1) / cps;  // runs part, part + cps, ...
+    const int tmax = (runs_here * kRun + kSampleBlock - 1) / kSampleBlock;
+    U v[PER];
 #pragma unroll
     for (int t = 0; t < PER; ++t) {
       const int slot = t * kSampleBlock + threadIdx.x;  // (run-in-part, lane)
-      const int run = (slot / kRun) * kSampleCTAs + part, e = slot % kRun;
-      const int s = run * kRun + e;
+      const int run = (slot / kRun) * cps + part, e = slot % kRun;
       const int64_t pos = (int64_t)run * stride + (stride - kRun) / 2 + e;
-      if (run < nruns && pos < p.len) samp[s] = (W)to_code_x<KIND>(__ldg(rowp + pos), xmask);
+      if (t < tmax && run < nruns && pos < p.len) v[t] = __ldg(rowp + pos);
+    }
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+      const int slot = t * kSampleBlock + threadIdx.x;
+      const int run = (slot / kRun) * cps + part, e = slot % kRun;
+      const int64_t pos = (int64_t)run * stride + (stride - kRun) / 2 + e;
+      if (t < tmax && run < nruns && pos < p.len) samp[run * kRun + e] = (W)to_code_x<KIND>(v[t], xmask);
     }
   }
-  __threadfence();
   __syncthreads();
-  if (threadIdx.x == 0) sh_last = (atomicAdd(&st->ticket, 1u) == (unsigned)(kSampleCTAs - 1));
+  if (threadIdx.x == 0) sh_last = (ticket_arrive(&st->ticket) == (unsigned)(cps - 1));
   __syncthreads();
   if (!sh_last) return;
-  __threadfence();
-  // phase 2 (last CTA of the row): the window from the sample order statistics
+  stamp(2);
+  // phase 2 (last CTA of the row): the window from the sample order statistics; the samples stay
+  // in registers (16 per thread)
+  constexpr int PER = kMaxSamples / kSampleBlock;
+  const int tv = (nsamp - (int)threadIdx.x + kSampleBlock - 1) / kSampleBlock;  // valid v[t]: t < tv
+  W v[PER];
+#pragma unroll
+  for (int t = 0; t < PER; ++t) v[t] = (t < tv) ? __ldcg(samp + t * kSampleBlock + threadIdx.x) : (W)0;
   {
-    constexpr int PER = kMaxSamples / kSampleBlock;  // all L2 loads in flight at once
-    W v[PER];
+    W lmin = ~(W)0, lmax = 0;
 #pragma unroll
     for (int t = 0; t < PER; ++t) {
-      const int s = t * kSampleBlock + threadIdx.x;
-      v[t] = (s < nsamp) ? __ldcg(samp + s) : (W)0;
+      if (t < tv) {
+        lmin = v[t] < lmin ? v[t] : lmin;
+        lmax = v[t] > lmax ? v[t] : lmax;
+      }
     }
 #pragma unroll
-    for (int t = 0; t < PER; ++t) {
-      const int s = t * kSampleBlock + threadIdx.x;
-      if (s < nsamp) codes[s] = v[t];
+    for (int o = 16; o > 0; o >>= 1) {
+      const W x = shfl(lmin, (threadIdx.x + o) & 31), y = shfl(lmax, (threadIdx.x + o) & 31);
+      lmin = x < lmin ? x : lmin;
+      lmax = y > lmax ? y : lmax;
     }
+    if ((threadIdx.x & 31) == 0) {
+      sh_red[threadIdx.x >> 5] = lmin;
+      sh_red[32 + (threadIdx.x >> 5)] = lmax;
+    }
+    if (threadIdx.x == 0) sh_cnt[2] = 0;
   }
   __syncthreads();
+  stamp(3);
   if (threadIdx.x == 0) st->ticket = 0;
   // expected sample rank of the K-th key and a 4-sigma (+8) margin of the binomial sample count
   // (measured sample counts are somewhat over-dispersed): a miss only costs the fallback, never
@@ -422,9 +529,36 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
     if (threadIdx.x == 0) st->win_state = 0;
     return;
   }
+  W smin = sh_red[0], smax = sh_red[32];
+#pragma unroll 8
+  for (int i = 1; i < kSampleBlock / 32; ++i) {
+    smin = sh_red[i] < smin ? sh_red[i] : smin;
+    smax = sh_red[32 + i] > smax ? sh_red[32 + i] : smax;
+  }
+  const W diff = smin ^ smax;
+  const int hb = diff ? (8 * (int)sizeof(W) - (sizeof(W) == 8 ? __clzll((long long)diff) : __clz((int)diff))) : 0;
+  stamp(5);
+  // no results below the window when rlo <= 0: everything up to hi is a candidate
   W lo, hi;
-  block_select_two<W>(codes, scratch, nsamp, rlo > 0 ? rlo : 0, rhi, KT<KIND>::R, hist, shw, sh_cnt, lo, hi);
-  if (rlo <= 0) lo = 0;  // no results below the window: everything up to hi is a candidate
+  block_select_two<W, PER>(v, tv, scratch, rlo <= 0 ? -1 : rlo, rhi, smin, hb, hist, wsum, shw, sh_cnt, lo, hi);
+  if (rlo <= 0) lo = 0;
+  stamp(6);
+  // Estimated window size from the sample (ties at hi included): a window that would overflow the
+  // candidate buffer (e.g. a row of equal keys) is not tried — the paper's passes run instead.
+  {
+    unsigned le = 0;
+#pragma unroll
+    for (int t = 0; t < PER; ++t) le += (t < tv) && v[t] <= hi && v[t] >= lo;
+    le = __reduce_add_sync(kFull, le);
+    if ((threadIdx.x & 31) == 0 && le) atomicAdd(&sh_cnt[2], (int)le);
+    __syncthreads();
+    const double est = (double)sh_cnt[2] / nsamp * (double)p.len;
+    if (est > 0.5 * (double)p.cap_rule) {
+      if (threadIdx.x == 0) st->win_state = 0;
+      return;
+    }
+  }
+  stamp(4);
   if (threadIdx.x == 0) {
     st->win_lo = lo;
     st->win_hi = hi;
@@ -473,33 +607,55 @@ cudaError_t launch_one(const GridParams& gp, unsigned grid, int q, int redo, cud
   return launch_pdl(pass_kernel<KIND, IdxT, DF, DH, HASIDX, TMA>, dim3(grid), dim3(kBlock), smem, s, gp, q, redo);
 }
 
+// one filter pass q >= 1 of variant v = DF * 3 + DH
+template <int KIND, typename IdxT, bool HASIDX, bool TMA>
+cudaError_t launch_grid_pass(const GridParams& gp, unsigned grid, int q, int v, cudaStream_t s) {
+  switch (v) {
+    case 1 * 3 + 1: return launch_one<KIND, IdxT, 1, 1, HASIDX, TMA>(gp, grid, q, 0, s);
+    case 1 * 3 + 2: return launch_one<KIND, IdxT, 1, 2, HASIDX, TMA>(gp, grid, q, 0, s);
+    case 2 * 3 + 2: return launch_one<KIND, IdxT, 2, 2, HASIDX, TMA>(gp, grid, q, 0, s);
+    case 2 * 3 + 0: return launch_one<KIND, IdxT, 2, 0, HASIDX, TMA>(gp, grid, q, 0, s);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
 template <int KIND, typename IdxT, bool HASIDX, bool TMA = false>
 cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, const Events& ev, cudaStream_t s,
-                               bool window_only = false) {
+                               int upto = 1 << 30) {
   const unsigned grid = (unsigned)((long long)batch * gp.cpr);
   int ie = 0;
   ev.record(ie++, s);
   if (nsamp > 0) {  // sample-guided window: sample, window pass (= pass 0 + filter), pass 0 over the window
     using W = std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long, unsigned>;
-    const size_t smem = (size_t)2 * kMaxSamples * 4;  // 8-byte keys: nsamp <= kMaxSamples / 2
+    const size_t smem = (size_t)kMaxSamples * 4;  // 8-byte keys: nsamp <= kMaxSamples / 2
     static const cudaError_t attr =
         cudaFuncSetAttribute(sample_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (attr != cudaSuccess) return attr;
-    cudaError_t es = launch_pdl(sample_kernel<KIND>, dim3((unsigned)(batch * kSampleCTAs)), dim3(kSampleBlock),
-                                (size_t)2 * nsamp * sizeof(W), s, gp, nsamp);
+    // CTAs per row: enough to spread a few rows' scattered loads over the SMs; one per row for
+    // batches (each CTA then keeps up to 16 loads per thread in flight)
+    const int cps = (int)std::max<int64_t>(1, std::min<int64_t>(kSampleCTAs, gp.nsms / batch));
+    cudaError_t es = launch_pdl(sample_kernel<KIND>, dim3((unsigned)(batch * cps)), dim3(kSampleBlock),
+                                (size_t)nsamp * sizeof(W), s, gp, nsamp, cps);
     if (es != cudaSuccess) return es;
     ev.record(ie++, s);
     cudaError_t e = launch_one<KIND, IdxT, 3, 0, HASIDX, TMA>(gp, grid, 0, 0, s);
     if (e != cudaSuccess) return e;
     ev.record(ie++, s);
-    if (window_only) return cudaGetLastError();
   }
-  for (int q = 0; q <= gp.P; ++q) {
+  for (int q = 0; q <= gp.P && q < upto; ++q) {
     const int DF = q == 0 ? 0 : (digit_of(q - 1, KT<KIND>::R, gp.IB).is_idx ? 2 : 1);
     const int DH = q == gp.P ? 0 : (digit_of(q, KT<KIND>::R, gp.IB).is_idx ? 2 : 1);
     const int v = DF * 3 + DH;
     cudaError_t e;
     const int redo = (q == 0 && nsamp > 0) ? 1 : 0;
+    if (TMA && nsamp > 0 && q >= 1) {  // window mode: the passes after it read the window buffer
+      GridParams gb = gp;
+      gb.cpr = gp.cpr_buf;
+      e = launch_grid_pass<KIND, IdxT, HASIDX, false>(gb, (unsigned)((long long)batch * gb.cpr), q, v, s);
+      if (e != cudaSuccess) return e;
+      ev.record(ie++, s);
+      continue;
+    }
     switch (v) {
       case 0 * 3 + 1: e = launch_one<KIND, IdxT, 0, 1, HASIDX, TMA>(gp, grid, q, redo, s); break;
       case 1 * 3 + 1: e = launch_one<KIND, IdxT, 1, 1, HASIDX, TMA>(gp, grid, q, 0, s); break;
@@ -524,12 +680,13 @@ cudaError_t launch_grid_kind(const SelectArgs& a, const Plan& pl, const GridPara
   const Events ev{a.events, a.n_events};
   if (a.in_idx) return launch_grid_passes<KIND, uint64_t, true>(gp, a.batch, 0, ev, s);
   cudaError_t e;
-  if (pl.idx64) e = launch_grid_passes<KIND, uint64_t, false>(gp, a.batch, pl.nsamp, ev, s, pl.tail != 0);
-  else if (pl.tma) e = launch_grid_passes<KIND, uint32_t, false, true>(gp, a.batch, pl.nsamp, ev, s, pl.tail != 0);
-  else e = launch_grid_passes<KIND, uint32_t, false>(gp, a.batch, pl.nsamp, ev, s, pl.tail != 0);
+  const int upto = pl.tail ? pl.tail_q : (1 << 30);
+  if (pl.idx64) e = launch_grid_passes<KIND, uint64_t, false>(gp, a.batch, pl.nsamp, ev, s, upto);
+  else if (pl.tma) e = launch_grid_passes<KIND, uint32_t, false, true>(gp, a.batch, pl.nsamp, ev, s, upto);
+  else e = launch_grid_passes<KIND, uint32_t, false>(gp, a.batch, pl.nsamp, ev, s, upto);
   if (e != cudaSuccess || !pl.tail) return e;
   e = launch_cluster_kind<KIND>(a, pl, ws, s, 1);
-  ev.record(3, s);
+  ev.record(3 + pl.tail_q, s);
   return e;
 }
 

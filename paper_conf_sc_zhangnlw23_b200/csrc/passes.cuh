@@ -20,6 +20,8 @@
 
 #include "device.cuh"
 #include "tma.cuh"
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
 
 namespace airtopk {
 
@@ -43,6 +45,52 @@ constexpr int kHistCopies = 4;
 constexpr int kDummyBin = kMaxBins;
 constexpr int kHistSlots = kMaxBins + 32;  // per copy; the dummy bin + padding
 
+// Conservative window prefilter for IEEE keys: true when some element of the tile may have
+// code <= whi, by a floating-point compare against hv = the key whose code is whi (select-min;
+// select-max mirrors it). x <=_total hv implies !(x >_fp hv): the IEEE total order refines the fp
+// order (-0 < +0 only in the former) and every compare with a NaN is false, so no result or window
+// member is missed; a false positive only sends the tile through the exact classification.
+template <int KIND, bool SELMIN, int N>
+__device__ __forceinline__ bool tile_maybe_le(const uint4 (&r)[N], uint32_t hv2) {
+  if constexpr (KIND == K_F32) {
+    const float h = __uint_as_float(hv2);
+    bool any = false;
+#pragma unroll
+    for (int u = 0; u < N; ++u) {
+      const uint32_t w[4] = {r[u].x, r[u].y, r[u].z, r[u].w};
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float x = __uint_as_float(w[e]);
+        any |= SELMIN ? !(x > h) : !(x < h);
+      }
+    }
+    return any;
+  } else {
+    unsigned acc = 0;
+#pragma unroll
+    for (int u = 0; u < N; ++u) {
+      const uint32_t w[4] = {r[u].x, r[u].y, r[u].z, r[u].w};
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        if constexpr (KIND == K_F16) {
+          const __half2 x = __halves2half2(__ushort_as_half((unsigned short)(w[e] & 0xffffu)),
+                                           __ushort_as_half((unsigned short)(w[e] >> 16)));
+          const __half2 h = __halves2half2(__ushort_as_half((unsigned short)(hv2 & 0xffffu)),
+                                           __ushort_as_half((unsigned short)(hv2 >> 16)));
+          acc |= SELMIN ? __hleu2_mask(x, h) : __hgeu2_mask(x, h);
+        } else {
+          const __nv_bfloat162 x = __halves2bfloat162(__ushort_as_bfloat16((unsigned short)(w[e] & 0xffffu)),
+                                                      __ushort_as_bfloat16((unsigned short)(w[e] >> 16)));
+          const __nv_bfloat162 h = __halves2bfloat162(__ushort_as_bfloat16((unsigned short)(hv2 & 0xffffu)),
+                                                      __ushort_as_bfloat16((unsigned short)(hv2 >> 16)));
+          acc |= SELMIN ? __hleu2_mask(x, h) : __hgeu2_mask(x, h);
+        }
+      }
+    }
+    return acc != 0;
+  }
+}
+
 // +1 on a shared-window address (no return value): red.shared.add, which the hardware aggregates
 // over lanes hitting the same address.
 __device__ __forceinline__ void shared_inc(unsigned addr) {
@@ -62,16 +110,14 @@ __host__ __device__ constexpr int hist_copies() {
   return (DF == 0 || DF == 3) ? 1 : (sizeof(U) + sizeof(IdxT) <= 8 ? kHistCopies : 2);
 }
 
-// Flush a warp queue: ONE global atomic reserves n slots, then coalesced stores. Out of line so the
-// streaming loop stays small (I-cache). mode 0: results (value bits + int64 index), 1: candidates.
+// Store a warp queue's n entries at [base, base + n) of the destination (coalesced); entries at or
+// beyond `limit` set the overflow flag instead. Out of line so the streaming loop stays small
+// (I-cache). mode 0: results (value bits + int64 index), 1: candidates (code + index).
 template <int KIND, typename IdxT>
-__device__ __noinline__ void wq_flush(const WarpQ<typename KT<KIND>::U, IdxT>* wq, int n, unsigned long long* counter,
+__device__ __noinline__ void wq_write(const WarpQ<typename KT<KIND>::U, IdxT>* wq, int n, unsigned long long base,
                                       unsigned long long limit, typename KT<KIND>::U* dst_code, void* dst_idx,
                                       int mode, bool sel_min, unsigned* err) {
   const int lane = threadIdx.x & 31;
-  unsigned long long base = 0;
-  if (lane == 0) base = atomicAdd(counter, (unsigned long long)n);
-  base = __shfl_sync(kFull, base, 0);
   for (int j = lane; j < n; j += 32) {
     const unsigned long long pos = base + j;
     if (pos < limit) {
@@ -86,6 +132,18 @@ __device__ __noinline__ void wq_flush(const WarpQ<typename KT<KIND>::U, IdxT>* w
       *err = mode == 0 ? 1u : 2u;
     }
   }
+}
+
+// Flush a full warp queue: ONE global atomic reserves n slots, then coalesced stores.
+template <int KIND, typename IdxT>
+__device__ __noinline__ void wq_flush(const WarpQ<typename KT<KIND>::U, IdxT>* wq, int n, unsigned long long* counter,
+                                      unsigned long long limit, typename KT<KIND>::U* dst_code, void* dst_idx,
+                                      int mode, bool sel_min, unsigned* err) {
+  const int lane = threadIdx.x & 31;
+  unsigned long long base = 0;
+  if (lane == 0) base = atomicAdd(counter, (unsigned long long)n);
+  base = __shfl_sync(kFull, base, 0);
+  wq_write<KIND, IdxT>(wq, n, base, limit, dst_code, dst_idx, mode, sel_min, err);
 }
 
 // Warp-collective append of the lanes with `pred` to a shared-memory queue (flushes when full).
@@ -162,7 +220,8 @@ struct PassCtx {
 
 // Runs the pass over this CTA's slice; all queues are flushed on return. Returns the number of
 // elements of the whole source (for the trace).
-template <int KIND, typename IdxT, int DF, int DH, bool HASIDX, int BLOCK, int HCOPIES = 0, bool TMA = false>
+template <int KIND, typename IdxT, int DF, int DH, bool HASIDX, int BLOCK, int HCOPIES = 0, bool TMA = false,
+          int BU = 4>
 __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT<KIND>::U, IdxT>& c) {
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;  // shifted-key width
@@ -210,6 +269,9 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
   // Filter classification of digit q-1 (Alg1 L15-22): win = result, cand = candidate for pass q.
   const W wlo = (W)c.lo, wspan = (W)c.span1;
   const W whi = (W)(wlo + wspan - 1);  // DF == 3: window [lo, hi]
+  // DF == 3 prefilter: the key whose code is whi (16-bit keys: in both halves)
+  const uint32_t hv2 = (sizeof(U) == 2) ? ((uint32_t)from_code<KIND>((U)whi, sel_min) * 0x10001u)
+                                        : (uint32_t)from_code<KIND>((U)whi, sel_min);
   auto classify = [&](U code, IdxT idx, bool valid, bool& win, bool& cand) {
     bool lt, eq;
     if constexpr (DF == 3) {  // sample-guided window
@@ -282,15 +344,22 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
       FlagT fl = 0;  // elements that must leave through the queues (results / stored candidates)
       if constexpr (DF == 3) {
         // window pass: results below the window -> output, window members -> candidate buffer and
-        // (slow path) the pass-1 histogram of the window members; a miss re-runs the paper's pass 1
+        // (slow path) the pass-1 histogram of the window members; a miss re-runs the paper's pass 1.
+        // Floating-point keys first take one conservative fp compare per element (two per HSETP2 for
+        // 16-bit keys): almost every tile holds neither result nor window member.
+        bool maybe = true;  // (no early return: the whole warp must reach the slow-path votes)
+        if constexpr (FULL && (KIND == K_F32 || KIND == K_F16 || KIND == K_BF16))
+          maybe = sel_min ? tile_maybe_le<KIND, true>(r, hv2) : tile_maybe_le<KIND, false>(r, hv2);
+        if (maybe) {
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
-          const bool valid = FULL || (vb + (int64_t)u * vs < vlim);
+          for (int u = 0; u < kUnroll; ++u) {
+            const bool valid = FULL || (vb + (int64_t)u * vs < vlim);
 #pragma unroll
-          for (int e = 0; e < VEC; ++e) {
-            const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
-            // result (code < lo) or window member (lo <= code <= hi): together simply code <= hi
-            if (valid && (W)code <= whi) fl |= (FlagT)1 << (u * VEC + e);
+            for (int e = 0; e < VEC; ++e) {
+              const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
+              // result (code < lo) or window member (lo <= code <= hi): together simply code <= hi
+              if (valid && (W)code <= whi) fl |= (FlagT)1 << (u * VEC + e);
+            }
           }
         }
       } else if constexpr (DF == 1 && DH == 1) {
@@ -507,7 +576,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
         shared_inc(hbase + 4u * (valid ? (unsigned)(((W)code >> shh) & hmask) : (unsigned)kDummyBin));
       }
     } else if constexpr (DF != 3) {
-      constexpr int BU = 4;  // coalesced entries per thread per iteration, all loads issued up front
+      // BU coalesced entries per thread per iteration, all loads issued up front
       for (unsigned long long base = e0; base < e1; base += (unsigned long long)BLOCK * BU) {
         U code[BU];
         IdxT idx[BU];
@@ -530,9 +599,38 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
     }
   }
   if constexpr (DF != 0) {
+    // final flush of the partial queues, aggregated over the CTA: one global atomic per CTA and
+    // destination instead of one per warp (same-address atomics serialise in L2: ~1 per ns)
+    constexpr int NW = BLOCK / 32;
+    static_assert(NW <= 32, "one warp scans the per-warp counts");
+    __shared__ unsigned long long s_base[2][NW];
+    __shared__ int s_n[2][NW];
     __syncwarp();
-    if (ocnt) wq_flush<KIND, IdxT>(c.oq, ocnt, c.outc, c.kk, c.ov, c.oi, 0, sel_min, c.err);
-    if (bcnt) wq_flush<KIND, IdxT>(c.bq, bcnt, c.bufc, c.capa, c.bco, c.bio, 1, sel_min, c.err);
+    if (lane == 0) {
+      s_n[0][tid >> 5] = ocnt;
+      s_n[1][tid >> 5] = bcnt;
+    }
+    __syncthreads();
+    if ((tid >> 5) == 0) {
+#pragma unroll
+      for (int mode = 0; mode < 2; ++mode) {
+        const unsigned x = (lane < NW) ? (unsigned)s_n[mode][lane] : 0u;
+        unsigned incl = x;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const unsigned y = __shfl_up_sync(kFull, incl, o);
+          if (lane >= o) incl += y;
+        }
+        const unsigned total = __shfl_sync(kFull, incl, 31);
+        unsigned long long b = 0;
+        if (lane == 0 && total) b = atomicAdd(mode ? c.bufc : c.outc, (unsigned long long)total);
+        b = __shfl_sync(kFull, b, 0);
+        if (lane < NW) s_base[mode][lane] = b + (incl - x);
+      }
+    }
+    __syncthreads();
+    if (ocnt) wq_write<KIND, IdxT>(c.oq, ocnt, s_base[0][tid >> 5], c.kk, c.ov, c.oi, 0, sel_min, c.err);
+    if (bcnt) wq_write<KIND, IdxT>(c.bq, bcnt, s_base[1][tid >> 5], c.capa, c.bco, c.bio, 1, sel_min, c.err);
   }
   if constexpr (DF == 3) {  // one atomic per warp: window-member extremes (the tail skips digits
                             // on which all members agree)
