@@ -70,8 +70,7 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
   using U = typename KT<KIND>::U;
   constexpr int HC = 1;
   extern __shared__ unsigned sh_hist[];  // kHistSlots counters
-  __shared__ WarpQ<U, IdxT> sh_oq[kCWarps];
-  __shared__ WarpQ<U, IdxT> sh_bq[kCWarps];
+  __shared__ WarpQ<U, IdxT> sh_wq[kCWarps];
   __shared__ ClusterShared cs;
   __shared__ unsigned sh_seg[kMaxBins];  // this CTA's merged bin segment
 
@@ -162,8 +161,8 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
       c.capa = (unsigned long long)p.cap_alloc;
       c.err = &st->error;
       c.hist = sh_hist;
-      c.oq = &sh_oq[warp];
-      c.bq = &sh_bq[warp];
+      c.ring = 0;
+      c.wq = &sh_wq[warp];
       const bool hist_on = c.do_hist || DF == 0;
       if (hist_on) {
         for (int i = tid; i < kHistSlots * HC; i += kCBlock) sh_hist[i] = 0;

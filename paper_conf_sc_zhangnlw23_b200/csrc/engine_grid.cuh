@@ -69,13 +69,8 @@ struct GridParams {
 constexpr int kBlock = 512;
 constexpr int kWarps = kBlock / 32;
 
-// dynamic shared memory of a pass kernel: [histogram copies][TMA warp rings][ring mbarriers]
-template <int HC>
-constexpr size_t tma_ring_offset() { return ((size_t)kHistSlots * 4 * HC + 127) / 128 * 128; }
-template <int KIND>
-constexpr size_t tma_ring_bytes() { return (size_t)kWarps * kTmaStages * 32 * kUnroll * 16; }
 #ifndef AIRTOPK_MINB
-#define AIRTOPK_MINB 3
+#define AIRTOPK_MINB 2
 #endif
 constexpr int kMinBlocks = AIRTOPK_MINB;
 constexpr int kMinBlocksFilter = AIRTOPK_SLOW_REG ? 2 : AIRTOPK_MINB;
@@ -94,8 +89,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   constexpr int HC = hist_copies<KIND, IdxT, DF>();
 
   extern __shared__ unsigned sh_hist[];  // kHistSlots * HC counters (dynamic: may exceed 48 KB)
-  __shared__ WarpQ<U, IdxT> sh_oq[HAS_Q ? kWarps : 1];
-  __shared__ WarpQ<U, IdxT> sh_bq[(HAS_Q && (DH != 0 || DF == 3)) ? kWarps : 1];  // candidate queues
+  __shared__ WarpQ<U, IdxT> sh_wq[HAS_Q ? kWarps : 1];  // per-warp tagged result / candidate queues
   __shared__ unsigned long long sh_tmp[kWarps];
   __shared__ ScanResult sh_res;
   __shared__ int sh_last;
@@ -155,9 +149,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.err = &st->error;
   c.hist = sh_hist;
   c.ring = smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>();
-  c.bars = c.ring + (unsigned)tma_ring_bytes<KIND>();
-  c.oq = &sh_oq[HAS_Q ? warp : 0];
-  c.bq = &sh_bq[(HAS_Q && (DH != 0 || DF == 3)) ? warp : 0];
+  c.wq = &sh_wq[HAS_Q ? warp : 0];
 
   const bool hist_on = c.do_hist || DF == 0 || DF == 3;
   if (hist_on) {
@@ -594,8 +586,7 @@ struct Events {
 template <int KIND, typename IdxT, int DF, int DH, bool TMA = false>
 constexpr size_t hist_smem_bytes() {
   constexpr int HC = hist_copies<KIND, IdxT, DF>();
-  return TMA ? tma_ring_offset<HC>() + tma_ring_bytes<KIND>() + (size_t)kWarps * kTmaStages * 8
-             : (size_t)kHistSlots * 4 * HC;
+  return TMA ? tma_smem_bytes<HC>() : (size_t)kHistSlots * 4 * HC;
 }
 
 template <int KIND, typename IdxT, int DF, int DH, bool HASIDX, bool TMA>

@@ -5,14 +5,21 @@
 //   DF (digit filtered, Alg1 L15-22): results (digit < target) -> output V/I; candidates
 //       (digit == target) -> candidate buffer if C < N/alpha (L17-18);
 //   DH (digit histogrammed, L12-13 / L19-20): candidates counted in the shared histogram.
-// DF/DH: 0 none, 1 key digit, 2 index digit (the lowest-index tie-break digits).
+// DF/DH: 0 none, 1 key digit, 2 index digit (the lowest-index tie-break digits);
+// DF == 3 is the sample-guided window pass.
 //
-// B200 choices (measured): 4 x 128-bit ld.global.nc.L1::no_allocate per
-// thread in flight; per-element work is 3-4 integer ops and a predicated shared atomic
-// (ATOMS.POPC.INC aggregates equal addresses within a warp); results/candidates, rare in most
-// passes, leave through per-warp shared queues flushed with one global atomic per 64 entries and
-// coalesced stores; the flagged element is re-read from L2 in the slow path so the tile registers
-// die early (40 registers -> 3 CTAs x 512 threads per SM, no spills).
+// B200 choices (measured, tools/microbench_stream.cu):
+//   * input streaming either by 4 x 128-bit ld.global.nc.L1::no_allocate per thread (register
+//     path) or through a per-CTA ring of 16 KiB bulk copies (cp.async.bulk, TMA engine) filled by
+//     one thread and consumed by all warps (full / empty mbarriers). Few large bulk copies keep
+//     ~190 KiB per SM in flight; many small per-warp copies measured 7-50 % slower;
+//   * per element, the fast path is a few integer ops: the histogram passes add a predicated
+//     shared atomic (hardware-aggregated for equal addresses), the window pass ONE compare of the
+//     raw key bits against a transformed threshold (exact, no key transform needed);
+//   * flagged elements (results / candidates; ~1 per warp tile in the window pass of c3) leave
+//     through ONE tagged queue per warp: a warp scan of the per-lane flag counts places every
+//     lane's flagged elements at once, the tag (result / candidate / drop) is set on the way in,
+//     and a full queue is flushed with one global atomic per destination and coalesced stores.
 #pragma once
 
 #include <algorithm>
@@ -20,23 +27,31 @@
 
 #include "device.cuh"
 #include "tma.cuh"
-#include <cuda_bf16.h>
-#include <cuda_fp16.h>
 
 namespace airtopk {
 
 #ifndef AIRTOPK_SLOW_REG
-#define AIRTOPK_SLOW_REG 0
+#define AIRTOPK_SLOW_REG 1  // register path: flagged elements re-read from the tile registers (1) or L2 (0)
 #endif
 #ifndef AIRTOPK_PREFETCH
-#define AIRTOPK_PREFETCH 0
+#define AIRTOPK_PREFETCH 0  // register path: issue the next tile's loads before classifying this one
 #endif
 #ifndef AIRTOPK_UNROLL
 #define AIRTOPK_UNROLL 4
 #endif
+#ifndef AIRTOPK_TMA_STAGES
+#define AIRTOPK_TMA_STAGES 12
+#endif
+#ifndef AIRTOPK_TMA_CHUNK
+#define AIRTOPK_TMA_CHUNK 32768
+#endif
 constexpr int kUnroll = AIRTOPK_UNROLL;
-constexpr int kQCap = 64;
-constexpr int kTmaStages = 4;  // per-warp ring depth of the bulk-copy streaming loop
+constexpr int kTmaStages = AIRTOPK_TMA_STAGES;       // max ring depth of the bulk-copy streaming loop
+constexpr unsigned kTmaChunk = AIRTOPK_TMA_CHUNK;    // bytes per bulk copy (one ring stage)
+// dynamic + static shared memory per CTA is capped at 227 KiB; the static part (queues, scan
+// scratch) of the grid pass kernel stays below 20 KiB
+constexpr size_t kSmemCap = 232448;
+constexpr size_t kStaticSmemReserve = 20480;
 // Copies of the shared histogram in the filter passes: lane l counts into copy l % kHistCopies
 // (interleaved bin-major so copies of one bin sit in different banks); cuts the same-address
 // serialisation of shared atomics when many lanes hit a few bins (radix-adversarial passes).
@@ -45,51 +60,17 @@ constexpr int kHistCopies = 4;
 constexpr int kDummyBin = kMaxBins;
 constexpr int kHistSlots = kMaxBins + 32;  // per copy; the dummy bin + padding
 
-// Conservative window prefilter for IEEE keys: true when some element of the tile may have
-// code <= whi, by a floating-point compare against hv = the key whose code is whi (select-min;
-// select-max mirrors it). x <=_total hv implies !(x >_fp hv): the IEEE total order refines the fp
-// order (-0 < +0 only in the former) and every compare with a NaN is false, so no result or window
-// member is missed; a false positive only sends the tile through the exact classification.
-template <int KIND, bool SELMIN, int N>
-__device__ __forceinline__ bool tile_maybe_le(const uint4 (&r)[N], uint32_t hv2) {
-  if constexpr (KIND == K_F32) {
-    const float h = __uint_as_float(hv2);
-    bool any = false;
-#pragma unroll
-    for (int u = 0; u < N; ++u) {
-      const uint32_t w[4] = {r[u].x, r[u].y, r[u].z, r[u].w};
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const float x = __uint_as_float(w[e]);
-        any |= SELMIN ? !(x > h) : !(x < h);
-      }
-    }
-    return any;
-  } else {
-    unsigned acc = 0;
-#pragma unroll
-    for (int u = 0; u < N; ++u) {
-      const uint32_t w[4] = {r[u].x, r[u].y, r[u].z, r[u].w};
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        if constexpr (KIND == K_F16) {
-          const __half2 x = __halves2half2(__ushort_as_half((unsigned short)(w[e] & 0xffffu)),
-                                           __ushort_as_half((unsigned short)(w[e] >> 16)));
-          const __half2 h = __halves2half2(__ushort_as_half((unsigned short)(hv2 & 0xffffu)),
-                                           __ushort_as_half((unsigned short)(hv2 >> 16)));
-          acc |= SELMIN ? __hleu2_mask(x, h) : __hgeu2_mask(x, h);
-        } else {
-          const __nv_bfloat162 x = __halves2bfloat162(__ushort_as_bfloat16((unsigned short)(w[e] & 0xffffu)),
-                                                      __ushort_as_bfloat16((unsigned short)(w[e] >> 16)));
-          const __nv_bfloat162 h = __halves2bfloat162(__ushort_as_bfloat16((unsigned short)(hv2 & 0xffffu)),
-                                                      __ushort_as_bfloat16((unsigned short)(hv2 >> 16)));
-          acc |= SELMIN ? __hleu2_mask(x, h) : __hgeu2_mask(x, h);
-        }
-      }
-    }
-    return acc != 0;
-  }
+template <int HC>
+constexpr size_t tma_ring_offset() { return ((size_t)kHistSlots * 4 * HC + 127) / 128 * 128; }
+template <int HC>
+constexpr int tma_stages() {
+  const size_t avail = kSmemCap - kStaticSmemReserve - tma_ring_offset<HC>() - 512;
+  const size_t s = avail / kTmaChunk;
+  return (int)(s < (size_t)kTmaStages ? s : (size_t)kTmaStages);
 }
+// dynamic shared memory of a TMA pass: [histogram copies][ring stages][full bars][empty bars]
+template <int HC>
+constexpr size_t tma_smem_bytes() { return tma_ring_offset<HC>() + (size_t)tma_stages<HC>() * (kTmaChunk + 16); }
 
 // +1 on a shared-window address (no return value): red.shared.add, which the hardware aggregates
 // over lanes hitting the same address.
@@ -97,11 +78,13 @@ __device__ __forceinline__ void shared_inc(unsigned addr) {
   asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(addr) : "memory");
 }
 
+// Per-warp queue of flagged elements. tag: 0 result (-> V, I), 1 candidate (-> buffer), 2 dropped.
 template <typename U, typename IdxT>
 struct WarpQ {
-  static constexpr int kCap = (sizeof(U) + sizeof(IdxT) <= 8) ? kQCap : kQCap / 2;
+  static constexpr int kCap = (sizeof(U) + sizeof(IdxT) <= 8) ? 128 : 64;
   U code[kCap];
   IdxT idx[kCap];
+  unsigned char tag[kCap];
 };
 
 template <int KIND, typename IdxT, int DF>
@@ -110,77 +93,69 @@ __host__ __device__ constexpr int hist_copies() {
   return (DF == 0 || DF == 3) ? 1 : (sizeof(U) + sizeof(IdxT) <= 8 ? kHistCopies : 2);
 }
 
-// Store a warp queue's n entries at [base, base + n) of the destination (coalesced); entries at or
-// beyond `limit` set the overflow flag instead. Out of line so the streaming loop stays small
-// (I-cache). mode 0: results (value bits + int64 index), 1: candidates (code + index).
+// Store the n queued entries of a warp: results at out[br ...], candidates at buf[bc ...], in queue
+// order (coalesced). Entries beyond a destination's limit set the error flag instead.
 template <int KIND, typename IdxT>
-__device__ __noinline__ void wq_write(const WarpQ<typename KT<KIND>::U, IdxT>* wq, int n, unsigned long long base,
-                                      unsigned long long limit, typename KT<KIND>::U* dst_code, void* dst_idx,
-                                      int mode, bool sel_min, unsigned* err) {
+__device__ __noinline__ void wq_write(const WarpQ<typename KT<KIND>::U, IdxT>* wq, int n, unsigned long long br,
+                                      unsigned long long bc, typename KT<KIND>::U* ov, int64_t* oi,
+                                      unsigned long long kk, typename KT<KIND>::U* bco, IdxT* bio,
+                                      unsigned long long capa, bool sel_min, unsigned* err) {
   const int lane = threadIdx.x & 31;
-  for (int j = lane; j < n; j += 32) {
-    const unsigned long long pos = base + j;
-    if (pos < limit) {
-      if (mode == 0) {
-        dst_code[pos] = from_code<KIND>(wq->code[j], sel_min);
-        ((int64_t*)dst_idx)[pos] = (int64_t)wq->idx[j];
+  const unsigned lt = lanemask_lt();
+  for (int j0 = 0; j0 < n; j0 += 32) {
+    const int j = j0 + lane;
+    const int tg = (j < n) ? (int)wq->tag[j] : 2;
+    const unsigned mr = __ballot_sync(kFull, tg == 0), mc = __ballot_sync(kFull, tg == 1);
+    if (tg == 0) {
+      const unsigned long long pos = br + __popc(mr & lt);
+      if (pos < kk) {
+        ov[pos] = from_code<KIND>(wq->code[j], sel_min);
+        oi[pos] = (int64_t)wq->idx[j];
       } else {
-        dst_code[pos] = wq->code[j];
-        ((IdxT*)dst_idx)[pos] = wq->idx[j];
+        *err |= 1u;
       }
-    } else {
-      *err = mode == 0 ? 1u : 2u;
+    } else if (tg == 1) {
+      const unsigned long long pos = bc + __popc(mc & lt);
+      if (pos < capa) {
+        bco[pos] = wq->code[j];
+        bio[pos] = wq->idx[j];
+      } else {
+        *err |= 2u;
+      }
     }
+    br += __popc(mr);
+    bc += __popc(mc);
   }
 }
 
-// Flush a full warp queue: ONE global atomic reserves n slots, then coalesced stores.
-template <int KIND, typename IdxT>
-__device__ __noinline__ void wq_flush(const WarpQ<typename KT<KIND>::U, IdxT>* wq, int n, unsigned long long* counter,
-                                      unsigned long long limit, typename KT<KIND>::U* dst_code, void* dst_idx,
-                                      int mode, bool sel_min, unsigned* err) {
+// Counts of results (low 16 bits) and candidates (high 16 bits) among a warp's n queued entries.
+template <typename U, typename IdxT>
+__device__ __forceinline__ unsigned wq_counts(const WarpQ<U, IdxT>* wq, int n) {
   const int lane = threadIdx.x & 31;
-  unsigned long long base = 0;
-  if (lane == 0) base = atomicAdd(counter, (unsigned long long)n);
-  base = __shfl_sync(kFull, base, 0);
-  wq_write<KIND, IdxT>(wq, n, base, limit, dst_code, dst_idx, mode, sel_min, err);
+  unsigned nr = 0, nc = 0;
+  for (int j0 = 0; j0 < n; j0 += 32) {
+    const int j = j0 + lane;
+    const int tg = (j < n) ? (int)wq->tag[j] : 2;
+    nr += __popc(__ballot_sync(kFull, tg == 0));
+    nc += __popc(__ballot_sync(kFull, tg == 1));
+  }
+  return nr | (nc << 16);
 }
 
-// Warp-collective append of the lanes with `pred` to a shared-memory queue (flushes when full).
+// Flush a full warp queue: ONE global atomic per destination reserves the slots, then coalesced
+// stores (wq_write stays out of line: I-cache; inlining this part avoids call-clobber spills).
 template <int KIND, typename IdxT>
-__device__ __forceinline__ void wq_push(WarpQ<typename KT<KIND>::U, IdxT>* wq, int& cnt, bool pred,
-                                        typename KT<KIND>::U code, IdxT idx, unsigned long long* counter,
-                                        unsigned long long limit, typename KT<KIND>::U* dst_code, void* dst_idx,
-                                        int mode, bool sel_min, unsigned* err) {
-  const unsigned m = __ballot_sync(kFull, pred);
-  if (!m) return;
-  const int n = __popc(m);
-  if (cnt + n > WarpQ<typename KT<KIND>::U, IdxT>::kCap) {
-    __syncwarp();
-    wq_flush<KIND, IdxT>(wq, cnt, counter, limit, dst_code, dst_idx, mode, sel_min, err);
-    cnt = 0;
-    __syncwarp();
-  }
-  if (pred) {
-    const int pos = cnt + __popc(m & lanemask_lt());
-    wq->code[pos] = code;
-    wq->idx[pos] = idx;
-  }
-  cnt += n;
-}
-
-// Element b (0 .. kUnroll*VEC-1) of a thread's tile registers, selected without local memory.
-template <typename U>
-__device__ __forceinline__ U tile_elem(const uint4 (&r)[kUnroll], int b) {
-  constexpr int VEC = 16 / sizeof(U);
-  const int u = b / VEC, e = b % VEC;
-  uint4 v = r[0];
-#pragma unroll
-  for (int i = 1; i < kUnroll; ++i) v = (u == i) ? r[i] : v;
-  U out = vec_elem<U>(v, 0);
-#pragma unroll
-  for (int i = 1; i < VEC; ++i) out = (e == i) ? vec_elem<U>(v, i) : out;
-  return out;
+__device__ __forceinline__ void wq_flush(const WarpQ<typename KT<KIND>::U, IdxT>* wq, int n, unsigned long long* outc,
+                                      unsigned long long* bufc, typename KT<KIND>::U* ov, int64_t* oi,
+                                      unsigned long long kk, typename KT<KIND>::U* bco, IdxT* bio,
+                                      unsigned long long capa, bool sel_min, unsigned* err) {
+  const int lane = threadIdx.x & 31;
+  const unsigned cnt = wq_counts(wq, n);
+  unsigned long long b = 0;
+  if (lane == 0 && (cnt & 0xffffu)) b = atomicAdd(outc, (unsigned long long)(cnt & 0xffffu));
+  if (lane == 1 && (cnt >> 16)) b = atomicAdd(bufc, (unsigned long long)(cnt >> 16));
+  const unsigned long long br = __shfl_sync(kFull, b, 0), bc = __shfl_sync(kFull, b, 1);
+  wq_write<KIND, IdxT>(wq, n, br, bc, ov, oi, kk, bco, bio, capa, sel_min, err);
 }
 
 // Everything one pass of one row needs (built by the engine from its copy of the row state).
@@ -213,21 +188,22 @@ struct PassCtx {
   unsigned long long* wnmin;     // DF == 3: atomicMax of ~code / code over the window members
   unsigned long long* wmax;
   unsigned* hist;  // shared, kMaxBins * hist_copies() counters, zeroed by the caller
-  unsigned ring, bars;  // TMA streaming: shared-window addresses of the warp rings and their mbarriers
-  WarpQ<U, IdxT>* oq;
-  WarpQ<U, IdxT>* bq;
+  unsigned ring;   // TMA streaming: shared-window address of the ring (after the histogram copies)
+  WarpQ<U, IdxT>* wq;
 };
 
-// Runs the pass over this CTA's slice; all queues are flushed on return. Returns the number of
+// Runs the pass over this CTA's slice; the queues are flushed on return. Returns the number of
 // elements of the whole source (for the trace).
 template <int KIND, typename IdxT, int DF, int DH, bool HASIDX, int BLOCK, int HCOPIES = 0, bool TMA = false,
           int BU = 4>
 __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT<KIND>::U, IdxT>& c) {
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;  // shifted-key width
+  using Q = WarpQ<U, IdxT>;
   constexpr int VEC = 16 / sizeof(U);
   constexpr int HC = HCOPIES > 0 ? HCOPIES : hist_copies<KIND, IdxT, DF>();  // histogram copies
-  const int tid = threadIdx.x, lane = tid & 31;
+  constexpr int NW = BLOCK / 32;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
 
   const int shh = c.dh.shift;
   const unsigned hmask = (1u << c.dh.width) - 1u;
@@ -257,21 +233,27 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
   // shared-window address of this lane's histogram copy (c.hist is the dynamic smem base)
   const unsigned hbase = (unsigned)__cvta_generic_to_shared(c.hist) + ((HC > 1) ? (unsigned)(lane % HC) * 4u : 0u);
   const U xmask = sel_min ? (U)0 : (U)~(U)0;
-  int ocnt = 0, bcnt = 0;
   W wlo_seen = ~(W)0, whi_seen = 0;  // DF == 3: extremes of this thread's window members
 
-  auto push_out = [&](bool pred, U code, IdxT idx) {
-    wq_push<KIND, IdxT>(c.oq, ocnt, pred, code, idx, c.outc, c.kk, c.ov, c.oi, 0, sel_min, c.err);
-  };
-  auto push_buf = [&](bool pred, U code, IdxT idx) {
-    wq_push<KIND, IdxT>(c.bq, bcnt, pred, code, idx, c.bufc, c.capa, c.bco, c.bio, 1, sel_min, c.err);
-  };
-  // Filter classification of digit q-1 (Alg1 L15-22): win = result, cand = candidate for pass q.
+  // Window [lo, hi] (DF == 3). code <= hi is tested on the RAW key bits b as (b ^ wx) <= hi: for
+  // IEEE keys with sign bit S, code(b) <= hi <=> b ^ S <= hi when hi >= S (select-min; the
+  // threshold key is non-negative, every negative key qualifies), <=> ~b <= hi when hi < S; the
+  // select-max and unsigned cases are the complements.
   const W wlo = (W)c.lo, wspan = (W)c.span1;
-  const W whi = (W)(wlo + wspan - 1);  // DF == 3: window [lo, hi]
-  // DF == 3 prefilter: the key whose code is whi (16-bit keys: in both halves)
-  const uint32_t hv2 = (sizeof(U) == 2) ? ((uint32_t)from_code<KIND>((U)whi, sel_min) * 0x10001u)
-                                        : (uint32_t)from_code<KIND>((U)whi, sel_min);
+  const W whi = (W)(wlo + wspan - 1);
+  W wx = 0;
+  if constexpr (DF == 3) {
+    constexpr W S = (W)((W)1 << (KT<KIND>::R - 1));
+    constexpr W ones = (W)(~(U)0);
+    if constexpr (KT<KIND>::IEEE) {
+      if (sel_min) wx = (whi >= S) ? S : ones;
+      else wx = (whi < S) ? (W)(ones ^ S) : (W)0;
+    } else {
+      wx = sel_min ? (W)0 : ones;
+    }
+  }
+
+  // Filter classification of digit q-1 (Alg1 L15-22): win = result, cand = candidate for pass q.
   auto classify = [&](U code, IdxT idx, bool valid, bool& win, bool& cand) {
     bool lt, eq;
     if constexpr (DF == 3) {  // sample-guided window
@@ -292,14 +274,50 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
     cand = valid && !emit_all && eq;
   };
   // Alg1 L19-20. Non-candidates count into a dummy bin instead of branching: a warp-uniform address
-  // is aggregated by the shared atomic unit (ATOMS.POPC.INC), so the common "no candidate" case is
-  // one cheap atomic and no divergence.
+  // is aggregated by the shared atomic unit, so the common "no candidate" case is one cheap atomic
+  // and no divergence.
   auto hist_cand = [&](U code, IdxT idx, bool cand) {
     unsigned d;
     if constexpr (DH == 2) d = (unsigned)(idx >> shh) & hmask;
     else d = (unsigned)((W)code >> shh) & hmask;
     d = (cand && do_hist) ? d : (unsigned)kDummyBin;
     shared_inc(hbase + d * (HC * 4));
+  };
+
+  // ---- the warp's tagged queue ----
+  Q* const wq = c.wq;
+  int qcnt = 0;
+  auto flush_full = [&]() {
+    __syncwarp();
+    wq_flush<KIND, IdxT>(wq, qcnt, c.outc, c.bufc, c.ov, c.oi, c.kk, c.bco, c.bio, c.capa, sel_min, c.err);
+    qcnt = 0;
+    __syncwarp();
+  };
+  // one element per lane (all lanes call): tag 0 result, 1 candidate
+  auto push1 = [&](bool pred, int tag, U code, IdxT idx) {
+    const unsigned m = __ballot_sync(kFull, pred);
+    if (!m) return;
+    const int n = __popc(m);
+    if (qcnt + n > Q::kCap) flush_full();
+    if (pred) {
+      const int pos = qcnt + __popc(m & lanemask_lt());
+      wq->code[pos] = code;
+      wq->idx[pos] = idx;
+      wq->tag[pos] = (unsigned char)tag;
+    }
+    qcnt += n;
+  };
+  auto tag_of = [&](U code, IdxT idx) -> int {
+    bool w, cd;
+    classify(code, idx, true, w, cd);
+    if constexpr (DF == 3) {
+      if (cd) {  // window member: extremes + the pass-1 digit histogram of the window buffer
+        wlo_seen = ((W)code < wlo_seen) ? (W)code : wlo_seen;
+        whi_seen = ((W)code > whi_seen) ? (W)code : whi_seen;
+        shared_inc(hbase + 4u * (unsigned)((W)code >> shh));
+      }
+    }
+    return w ? 0 : ((cd && store) ? 1 : 2);
   };
 
   unsigned long long nread;
@@ -318,18 +336,67 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
       else return (IdxT)pos;
     };
 
-    // One thread's tile: kUnroll 16-byte vectors at vector indices vb + u*BLOCK. FULL: all valid.
-    // vs = distance (in 16-byte vectors) between a thread's kUnroll vectors: BLOCK for CTA tiles read
-    // with registers, 32 for warp tiles staged through shared memory by the bulk-copy engine
-    // sstage: shared-window address of the warp's staged tile (TMA path) or 0 (register path): the
-    // slow path then re-reads a flagged element from shared memory instead of L2
-    auto process_tile = [&](const uint4 (&r)[kUnroll], int64_t vb, int64_t vlim, auto full_tag, int64_t vs,
-                            unsigned sstage) {
+    // Flagged elements of a tile -> the warp queue. Lane-local flags fl (bit b = element b of the
+    // lane's tile); a warp scan of the flag counts gives every lane its queue slots, so the usual
+    // case (a handful of flagged elements per warp tile) is one scan and one short loop per lane.
+    // get(b, pos) returns the raw key of element b (shared-memory stage, registers or L2).
+    auto drain = [&](auto fl, int64_t vb, int64_t vs, auto get) {
+      using FlagT = decltype(fl);
+      // usual case, at most one flagged element per lane: slots from one ballot (no scan chain)
+      if (!__any_sync(kFull, (fl & (fl - 1)) != 0)) {
+        const unsigned m = __ballot_sync(kFull, fl != 0);
+        const int total = __popc(m);
+        if (qcnt + total > Q::kCap) flush_full();
+        if (fl) {
+          const int qp = qcnt + __popc(m & lanemask_lt());
+          const int b = ((sizeof(FlagT) == 8) ? __ffsll((long long)fl) : __ffs((int)fl)) - 1;
+          const int64_t pos = head + (vb + (int64_t)(b / VEC) * vs) * VEC + (b % VEC);
+          const U code = to_code_x<KIND>(get(b, pos), xmask);
+          const IdxT idx = index_of(pos);
+          wq->code[qp] = code;
+          wq->idx[qp] = idx;
+          wq->tag[qp] = (unsigned char)tag_of(code, idx);
+        }
+        qcnt += total;
+        return;
+      }
+      while (true) {
+        const int n = (sizeof(FlagT) == 8) ? __popcll((unsigned long long)fl) : __popc((unsigned)fl);
+        int incl = n;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int y = __shfl_up_sync(kFull, incl, o);
+          if (lane >= o) incl += y;
+        }
+        const int total = __shfl_sync(kFull, incl, 31);
+        int qp = qcnt + incl - n;
+        while (fl && qp < Q::kCap) {
+          const int b = ((sizeof(FlagT) == 8) ? __ffsll((long long)fl) : __ffs((int)fl)) - 1;
+          fl &= fl - 1;
+          const int64_t pos = head + (vb + (int64_t)(b / VEC) * vs) * VEC + (b % VEC);
+          const U code = to_code_x<KIND>(get(b, pos), xmask);
+          const IdxT idx = index_of(pos);
+          wq->code[qp] = code;
+          wq->idx[qp] = idx;
+          wq->tag[qp] = (unsigned char)tag_of(code, idx);
+          ++qp;
+        }
+        const bool fits = qcnt + total <= Q::kCap;
+        qcnt = fits ? qcnt + total : Q::kCap;
+        if (qcnt == Q::kCap) flush_full();
+        if (fits || !__any_sync(kFull, fl != 0)) break;
+      }
+    };
+
+    // One thread's tile: NV 16-byte vectors at vector indices vb + u*vs. FULL: all valid.
+    // sstage: shared-window address of the warp's staged tile (TMA path) or 0 (register path).
+    auto process_tile = [&](const auto& r, int64_t vb, int64_t vlim, auto full_tag, int64_t vs, unsigned sstage) {
       constexpr bool FULL = decltype(full_tag)::value;
+      constexpr int NV = (int)(sizeof(r) / sizeof(uint4));
       if constexpr (DF == 0) {
         // pass 1: the top digit needs no mask (code >> shh < 2^11)
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
+        for (int u = 0; u < NV; ++u) {
           const bool valid = FULL || (vb + (int64_t)u * vs < vlim);
 #pragma unroll
           for (int e = 0; e < VEC; ++e) {
@@ -339,196 +406,209 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
           }
         }
         return;
-      }
-      using FlagT = std::conditional_t<(kUnroll * VEC > 32), unsigned long long, unsigned>;
-      FlagT fl = 0;  // elements that must leave through the queues (results / stored candidates)
-      if constexpr (DF == 3) {
-        // window pass: results below the window -> output, window members -> candidate buffer and
-        // (slow path) the pass-1 histogram of the window members; a miss re-runs the paper's pass 1.
-        // Floating-point keys first take one conservative fp compare per element (two per HSETP2 for
-        // 16-bit keys): almost every tile holds neither result nor window member.
-        bool maybe = true;  // (no early return: the whole warp must reach the slow-path votes)
-        if constexpr (FULL && (KIND == K_F32 || KIND == K_F16 || KIND == K_BF16))
-          maybe = sel_min ? tile_maybe_le<KIND, true>(r, hv2) : tile_maybe_le<KIND, false>(r, hv2);
-        if (maybe) {
+      } else {
+        using FlagT = std::conditional_t<(NV * VEC > 32), unsigned long long, unsigned>;
+        FlagT fl = 0;  // elements that must leave through the queue (results / stored candidates)
+        if constexpr (DF == 3) {
+          // window pass: result (code < lo) or window member (lo <= code <= hi), together code <= hi,
+          // tested on the raw bits: the lane's minimum of b ^ wx (one xor + one min per element), the
+          // per-element flags only when the minimum hits (a few lanes per warp tile)
+          W m = ~(W)0;
 #pragma unroll
-          for (int u = 0; u < kUnroll; ++u) {
+          for (int u = 0; u < NV; ++u) {
+            const bool valid = FULL || (vb + (int64_t)u * vs < vlim);
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) {
+              const W t = (W)((W)vec_elem<U>(r[u], e) ^ wx);
+              m = (valid && t < m) ? t : m;
+            }
+          }
+          if (m <= whi) {
+#pragma unroll
+            for (int u = 0; u < NV; ++u) {
+              const bool valid = FULL || (vb + (int64_t)u * vs < vlim);
+#pragma unroll
+              for (int e = 0; e < VEC; ++e)
+                if (valid && (W)((W)vec_elem<U>(r[u], e) ^ wx) <= whi) fl |= (FlagT)1 << (u * VEC + e);
+            }
+          }
+        } else if constexpr (DF == 1 && DH == 1) {
+          // adjacent key digits: y = (code >> shh) - B places the elements whose higher digits match
+          // the prefix at [S, S + nb) and the results below S (see the derivation at kx_* above)
+#pragma unroll
+          for (int u = 0; u < NV; ++u) {
             const bool valid = FULL || (vb + (int64_t)u * vs < vlim);
 #pragma unroll
             for (int e = 0; e < VEC; ++e) {
               const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
-              // result (code < lo) or window member (lo <= code <= hi): together simply code <= hi
-              if (valid && (W)code <= whi) fl |= (FlagT)1 << (u * VEC + e);
+              const W y = ((W)code >> shh) - kx_B;
+              const unsigned d = (unsigned)min((W)(y - kx_S), (W)kDummyBin);
+              shared_inc(hbase + (valid ? d : (unsigned)kDummyBin) * (HC * 4u));
+              // result (y < S) or stored candidate / emit-all member (S <= y < S + nb): one compare
+              if (valid && y < kx_flag) fl |= (FlagT)1 << (u * VEC + e);
+            }
+          }
+        } else {
+#pragma unroll
+          for (int u = 0; u < NV; ++u) {
+            const int64_t v = vb + (int64_t)u * vs;
+            const bool valid = FULL || (v < vlim);
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) {
+              const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
+              IdxT idx = 0;
+              if constexpr (DF == 2 || DH == 2) {
+                // the index is needed to classify (DF == 2) or to histogram a candidate (DH == 2)
+                bool need = true;
+                if constexpr (HASIDX) need = (DF == 2) ? (code == fc) : (((W)code >> sf) == tc);
+                if (need && valid) idx = index_of(head + v * VEC + e);
+              }
+              bool win, cand;
+              classify(code, idx, valid, win, cand);
+              hist_cand(code, idx, cand);
+              if (win || (cand && store)) fl |= (FlagT)1 << (u * VEC + e);
             }
           }
         }
-      } else if constexpr (DF == 1 && DH == 1) {
-        // adjacent key digits: y = (code >> shh) - B places the elements whose higher digits match
-        // the prefix at [S, S + nb) and the results below S (see the derivation at kx_* below)
-#pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
-          const bool valid = FULL || (vb + (int64_t)u * vs < vlim);
-#pragma unroll
-          for (int e = 0; e < VEC; ++e) {
-            const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
-            const W y = ((W)code >> shh) - kx_B;
-            const unsigned d = (unsigned)min((W)(y - kx_S), (W)kDummyBin);
-            shared_inc(hbase + (valid ? d : (unsigned)kDummyBin) * (HC * 4u));
-            // result (y < S) or stored candidate / emit-all member (S <= y < S + nb): one compare
-            if (valid && y < kx_flag) fl |= (FlagT)1 << (u * VEC + e);
-          }
-        }
-      } else {
-#pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
-          const int64_t v = vb + (int64_t)u * vs;
-          const bool valid = FULL || (v < vlim);
-#pragma unroll
-          for (int e = 0; e < VEC; ++e) {
-            const U code = to_code_x<KIND>(vec_elem<U>(r[u], e), xmask);
-            IdxT idx = 0;
-            if constexpr (DF == 2 || DH == 2) {
-              // the index is needed to classify (DF == 2) or to histogram a candidate (DH == 2)
-              bool need = true;
-              if constexpr (HASIDX) need = (DF == 2) ? (code == fc) : (((W)code >> sf) == tc);
-              if (need && valid) idx = index_of(head + v * VEC + e);
-            }
-            bool win, cand;
-            classify(code, idx, valid, win, cand);
-            hist_cand(code, idx, cand);
-            if (win || (cand && store)) fl |= (FlagT)1 << (u * VEC + e);
-          }
-        }
-      }
-      // slow path (rare in most passes): results / candidates through the warp queues. The flagged
-      // element is re-read (an L2 hit: this warp just streamed it) and re-classified, so the tile
-      // registers die early.
-      while (__any_sync(kFull, fl != 0)) {
-        const bool has = fl != 0;
-        const int b = has ? ((sizeof(FlagT) == 8) ? __ffsll((long long)fl) : __ffs((int)fl)) - 1 : 0;
-        fl &= fl - 1;
-        const int64_t pos = head + (vb + (int64_t)(b / VEC) * vs) * VEC + (b % VEC);
-        U raw = 0;
-        if (has) {
+        if (__any_sync(kFull, fl != 0)) {
           if (TMA && sstage) {
-            const unsigned a = sstage + (unsigned)((((b / VEC) * 32 + lane) * 16) + (b % VEC) * (int)sizeof(U));
-            if constexpr (sizeof(U) == 2) { unsigned short t; asm volatile("ld.shared.u16 %0, [%1];" : "=h"(t) : "r"(a)); raw = (U)t; }
-            else if constexpr (sizeof(U) == 4) { unsigned t; asm volatile("ld.shared.u32 %0, [%1];" : "=r"(t) : "r"(a)); raw = (U)t; }
-            else { unsigned long long t; asm volatile("ld.shared.u64 %0, [%1];" : "=l"(t) : "r"(a)); raw = (U)t; }
+            drain(fl, vb, vs, [&](int b, int64_t) -> U {
+              const unsigned a = sstage + (unsigned)((((b / VEC) * 32 + lane) * 16) + (b % VEC) * (int)sizeof(U));
+              if constexpr (sizeof(U) == 2) { unsigned short t; asm volatile("ld.shared.u16 %0, [%1];" : "=h"(t) : "r"(a)); return (U)t; }
+              else if constexpr (sizeof(U) == 4) { unsigned t; asm volatile("ld.shared.u32 %0, [%1];" : "=r"(t) : "r"(a)); return (U)t; }
+              else { unsigned long long t; asm volatile("ld.shared.u64 %0, [%1];" : "=l"(t) : "r"(a)); return (U)t; }
+            });
           } else {
 #if AIRTOPK_SLOW_REG
-            raw = tile_elem<U>(r, b);
+            drain(fl, vb, vs, [&](int b, int64_t) -> U {
+              const int u = b / VEC, e = b % VEC;
+              uint4 v = r[0];
+#pragma unroll
+              for (int i = 1; i < NV; ++i) v = (u == i) ? r[i] : v;
+              U out = vec_elem<U>(v, 0);
+#pragma unroll
+              for (int i = 1; i < VEC; ++i) out = (e == i) ? vec_elem<U>(v, i) : out;
+              return out;
+            });
 #else
-            raw = __ldcg(rowp + pos);
+            drain(fl, vb, vs, [&](int, int64_t pos) -> U { return __ldcg(rowp + pos); });
 #endif
           }
         }
-        const U code = to_code_x<KIND>(raw, xmask);
-        const IdxT idx = has ? index_of(pos) : (IdxT)0;
-        bool w, cd;
-        classify(code, idx, has, w, cd);
-        if constexpr (DF == 3) {
-          if (cd) {  // window member: extremes + the pass-1 digit histogram of the window buffer
-            wlo_seen = ((W)code < wlo_seen) ? (W)code : wlo_seen;
-            whi_seen = ((W)code > whi_seen) ? (W)code : whi_seen;
-            shared_inc(hbase + 4u * (unsigned)((W)code >> shh));
-          }
-        }
-        push_out(w, code, idx);
-        if (store) push_buf(cd, code, idx);
       }
     };
 
-    // Grid-stride tile order: tile t (BLOCK*kUnroll 16-byte vectors, 32 KiB for 512 threads) goes to
-    // slice t mod nslices, so at any moment the CTAs of a row read one compact, advancing region of
-    // HBM. Measured on B200: zero DRAM over-fetch and 7.2-7.4 TB/s, vs 9% over-fetch and 6.3 TB/s
-    // when every CTA streams its own contiguous chunk (tools/microbench_hist.cu, profiles/).
-    // `reverse` walks the tiles backwards (odd passes consume the tail the previous pass left in L2).
     if constexpr (TMA) {
-      // Warp tiles of 32 x kUnroll 16-byte vectors (2 KiB for f32) in grid-stride order over all
-      // warps of the row's CTAs; each warp streams its tiles through its own NST-stage shared ring
-      // filled by the bulk-copy engine (lane 0 issues, the stage's mbarrier counts the bytes).
-      constexpr int NW = BLOCK / 32;
-      constexpr int64_t WT = 32 * kUnroll;
-      constexpr unsigned WT_BYTES = (unsigned)(WT * 16);
-      const int warp = tid >> 5;
-      const int64_t G = (int64_t)c.nslices * NW, g = (int64_t)c.slice * NW + warp;
-      const int64_t nwt = nvec / WT;
-      const int64_t mine = (nwt > g) ? (nwt - 1 - g) / G + 1 : 0;
-      auto wtile = [&](int64_t i) { return g + (c.reverse ? (mine - 1 - i) : i) * G; };
-      const unsigned ring = c.ring + (unsigned)warp * (unsigned)(kTmaStages * WT_BYTES);
-      const unsigned bars = c.bars + (unsigned)warp * (unsigned)(kTmaStages * 8);
-      if (lane == 0) {
-        for (int st = 0; st < kTmaStages; ++st) mbar_init(bars + 8u * st, 1);
+      // Per-CTA ring of NST stages of kTmaChunk bytes in grid-stride chunk order (chunk t -> CTA
+      // t mod nslices of the row): thread 0 issues the bulk copies (completion counted on the
+      // stage's full barrier), every warp consumes its NVT vectors per lane of a stage and arrives
+      // on the stage's empty barrier; thread 0 refills a stage once all warps released it (lagged
+      // by one iteration so it seldom waits).
+      constexpr int NST = tma_stages<HC>();
+      constexpr int NVT = (int)(kTmaChunk / 16 / BLOCK);
+      static_assert(NVT >= 1 && kTmaChunk % (16 * BLOCK) == 0, "chunk = BLOCK x NVT 16-byte vectors");
+      constexpr int64_t CV = (int64_t)BLOCK * NVT;  // vectors per chunk
+      const unsigned ring = c.ring;
+      const unsigned fullb = ring + NST * kTmaChunk, emptyb = fullb + 8u * NST;
+      const int64_t nch = nvec / CV;
+      const int64_t mine = (nch > c.slice) ? (nch - 1 - c.slice) / c.nslices + 1 : 0;
+      // chunk of iteration i: c0 + i * cstep (all index arithmetic incremental: no 64-bit divisions
+      // in the loop)
+      const int64_t c0 = c.reverse ? (int64_t)c.slice + (mine - 1) * c.nslices : (int64_t)c.slice;
+      const int64_t cstep = c.reverse ? -(int64_t)c.nslices : (int64_t)c.nslices;
+      const uint4* const src0 = vp + c0 * CV;
+      const int64_t sstep = cstep * CV;  // in 16-byte vectors
+      if (tid == 0) {
+        for (int st = 0; st < NST; ++st) {
+          mbar_init(fullb + 8u * st, 1);
+          mbar_init(emptyb + 8u * st, NW);
+        }
         fence_mbar_init();
-        for (int st = 0; st < kTmaStages && st < mine; ++st) {
-          mbar_arrive_expect_tx(bars + 8u * st, WT_BYTES);
-          bulk_g2s(ring + st * WT_BYTES, vp + wtile(st) * WT, WT_BYTES, bars + 8u * st);
+        for (int st = 0; st < NST && st < mine; ++st) {
+          mbar_arrive_expect_tx(fullb + 8u * st, kTmaChunk);
+          bulk_g2s(ring + st * kTmaChunk, src0 + st * sstep, kTmaChunk, fullb + 8u * st);
         }
       }
-      __syncwarp();
+      __syncthreads();
+      int st = 0, pst = NST - 1;    // stage of this / the previous iteration
+      unsigned ph = 0, pph = 1;     // their phase parities
+      int64_t vb = c0 * CV + (int64_t)warp * NVT * 32 + lane;
+      const uint4* refill = src0 + (int64_t)(NST - 1) * sstep;  // chunk of iteration i - 1 + NST
       for (int64_t i = 0; i < mine; ++i) {
-        const int st = (int)(i % kTmaStages);
-        mbar_wait(bars + 8u * st, (unsigned)((i / kTmaStages) & 1));
-        uint4 r[kUnroll];
-        const unsigned sbase = ring + st * WT_BYTES;
+        mbar_wait(fullb + 8u * st, ph);
+        const unsigned sw = ring + st * kTmaChunk + (unsigned)(warp * NVT * 32 * 16);  // this warp's part
+        uint4 r[NVT];
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) r[u] = lds128(sbase + (unsigned)((u * 32 + lane) * 16));
-        process_tile(r, wtile(i) * WT + lane, nvec, std::true_type{}, (int64_t)32, sbase);
+        for (int u = 0; u < NVT; ++u) r[u] = lds128(sw + (unsigned)((u * 32 + lane) * 16));
+        process_tile(r, vb, nvec, std::true_type{}, (int64_t)32, sw);
         __syncwarp();
-        if (lane == 0 && i + kTmaStages < mine) {  // refill the consumed stage (kTmaStages-1 in flight)
+        if (lane == 0) mbar_arrive(emptyb + 8u * st);
+        if (tid == 0 && i >= 1 && i - 1 + NST < mine) {  // refill the stage released one iteration ago
+          mbar_wait(emptyb + 8u * pst, pph);
           fence_proxy_async_smem();
-          mbar_arrive_expect_tx(bars + 8u * st, WT_BYTES);
-          bulk_g2s(sbase, vp + wtile(i + kTmaStages) * WT, WT_BYTES, bars + 8u * st);
+          mbar_arrive_expect_tx(fullb + 8u * pst, kTmaChunk);
+          bulk_g2s(ring + pst * kTmaChunk, refill, kTmaChunk, fullb + 8u * pst);
         }
+        refill += sstep;
+        pst = st;
+        pph = ph;
+        if (++st == NST) {
+          st = 0;
+          ph ^= 1u;
+        }
+        vb += sstep;
       }
-      if (nwt * WT < nvec && g == (nwt % G)) {  // the partial last warp tile
-        const int64_t vb = nwt * WT + lane;
-        uint4 r[kUnroll];
+      if (nch * CV < nvec && c.slice == (int)(nch % c.nslices)) {  // the partial last chunk
+        const int64_t vb = nch * CV + (int64_t)warp * NVT * 32 + lane;
+        uint4 r[NVT];
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
+        for (int u = 0; u < NVT; ++u) {
           const int64_t v = vb + (int64_t)u * 32;
           r[u] = (v < nvec) ? ldg_stream(vp + v) : make_uint4(0, 0, 0, 0);
         }
         process_tile(r, vb, nvec, std::false_type{}, (int64_t)32, 0u);
       }
     } else {
+      // Grid-stride tile order: tile t (BLOCK*kUnroll 16-byte vectors, 32 KiB for 512 threads) goes
+      // to slice t mod nslices, so at any moment the CTAs of a row read one compact, advancing region
+      // of HBM. Measured on B200: zero DRAM over-fetch and 7.2-7.4 TB/s, vs 9% over-fetch and 6.3
+      // TB/s when every CTA streams its own contiguous chunk (tools/microbench_hist.cu, profiles/).
+      // `reverse` walks the tiles backwards (odd passes consume the tail the previous pass left in L2).
       const int64_t tile = (int64_t)BLOCK * kUnroll;
       const int64_t ntiles = nvec / tile;
       const int64_t mine = (ntiles > c.slice) ? (ntiles - 1 - c.slice) / c.nslices + 1 : 0;
-  #if AIRTOPK_PREFETCH
+      const int64_t t0 = c.reverse ? (int64_t)c.slice + (mine - 1) * c.nslices : (int64_t)c.slice;
+      const int64_t vstep = (c.reverse ? -(int64_t)c.nslices : (int64_t)c.nslices) * tile;
+      int64_t vb = t0 * tile + tid;
+#if AIRTOPK_PREFETCH
       // software pipeline: the next tile's loads are in flight while this tile is classified
       if (mine > 0) {
-        auto tile_of = [&](int64_t i) { return (int64_t)c.slice + (c.reverse ? (mine - 1 - i) : i) * c.nslices; };
         uint4 r[kUnroll];
-        int64_t vb = tile_of(0) * tile + tid;
-  #pragma unroll
+#pragma unroll
         for (int u = 0; u < kUnroll; ++u) r[u] = ldg_stream(vp + vb + (int64_t)u * BLOCK);
         for (int64_t i = 0; i < mine; ++i) {
           uint4 nx[kUnroll];
-          const int64_t vbn = (i + 1 < mine) ? tile_of(i + 1) * tile + tid : vb;
-  #pragma unroll
-          for (int u = 0; u < kUnroll; ++u) nx[u] = ldg_stream(vp + vbn + (int64_t)u * BLOCK);
+          const int64_t vn = (i + 1 < mine) ? vb + vstep : vb;
+#pragma unroll
+          for (int u = 0; u < kUnroll; ++u) nx[u] = ldg_stream(vp + vn + (int64_t)u * BLOCK);
           process_tile(r, vb, nvec, std::true_type{}, (int64_t)BLOCK, 0u);
-  #pragma unroll
+#pragma unroll
           for (int u = 0; u < kUnroll; ++u) r[u] = nx[u];
-          vb = vbn;
+          vb = vn;
         }
       }
-  #else
-      for (int64_t i = 0; i < mine; ++i) {
-        const int64_t t = (int64_t)c.slice + (c.reverse ? (mine - 1 - i) : i) * c.nslices;
-        const int64_t vb = t * tile + tid;
+#else
+      for (int64_t i = 0; i < mine; ++i, vb += vstep) {
         uint4 r[kUnroll];
-  #pragma unroll
+#pragma unroll
         for (int u = 0; u < kUnroll; ++u) r[u] = ldg_stream(vp + vb + (int64_t)u * BLOCK);
         process_tile(r, vb, nvec, std::true_type{}, (int64_t)BLOCK, 0u);
       }
-  #endif
+#endif
       if (ntiles * tile < nvec && c.slice == (int)(ntiles % c.nslices)) {  // the partial last tile
         const int64_t vb = ntiles * tile + tid;
         uint4 r[kUnroll];
-  #pragma unroll
+#pragma unroll
         for (int u = 0; u < kUnroll; ++u) {
           const int64_t v = vb + (int64_t)u * BLOCK;
           r[u] = (v < nvec) ? ldg_stream(vp + v) : make_uint4(0, 0, 0, 0);
@@ -546,15 +626,8 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
         bool win, cand;
         classify(code, idx, valid, win, cand);
         if constexpr (DF != 3) hist_cand(code, idx, cand);
-        if constexpr (DF == 3) {
-          if (cand) {
-            wlo_seen = ((W)code < wlo_seen) ? (W)code : wlo_seen;
-            whi_seen = ((W)code > whi_seen) ? (W)code : whi_seen;
-            shared_inc(hbase + 4u * (unsigned)((W)code >> shh));
-          }
-        }
-        push_out(win, code, idx);
-        if (store) push_buf(cand, code, idx);
+        const int tg = (win || cand) ? tag_of(code, idx) : 2;
+        push1(tg != 2, tg, code, idx);
       }
     };
     for (int64_t hb = 0; hb < head; hb += BLOCK)
@@ -592,8 +665,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
           bool win, cand;
           classify(code[j], idx[j], valid, win, cand);
           hist_cand(code[j], idx[j], cand);
-          push_out(win, code[j], idx[j]);
-          if (store) push_buf(cand, code[j], idx[j]);
+          push1(win || (cand && store), win ? 0 : 1, code[j], idx[j]);
         }
       }
     }
@@ -601,36 +673,36 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
   if constexpr (DF != 0) {
     // final flush of the partial queues, aggregated over the CTA: one global atomic per CTA and
     // destination instead of one per warp (same-address atomics serialise in L2: ~1 per ns)
-    constexpr int NW = BLOCK / 32;
     static_assert(NW <= 32, "one warp scans the per-warp counts");
     __shared__ unsigned long long s_base[2][NW];
-    __shared__ int s_n[2][NW];
+    __shared__ unsigned s_n[NW];
     __syncwarp();
-    if (lane == 0) {
-      s_n[0][tid >> 5] = ocnt;
-      s_n[1][tid >> 5] = bcnt;
-    }
+    const unsigned cnt = wq_counts(wq, qcnt);
+    if (lane == 0) s_n[warp] = cnt;
     __syncthreads();
-    if ((tid >> 5) == 0) {
+    if (warp == 0) {
+      const unsigned x = (lane < NW) ? s_n[lane] : 0u;  // (results | candidates << 16) per warp
+      unsigned incl = x;
 #pragma unroll
-      for (int mode = 0; mode < 2; ++mode) {
-        const unsigned x = (lane < NW) ? (unsigned)s_n[mode][lane] : 0u;
-        unsigned incl = x;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const unsigned y = __shfl_up_sync(kFull, incl, o);
-          if (lane >= o) incl += y;
-        }
-        const unsigned total = __shfl_sync(kFull, incl, 31);
-        unsigned long long b = 0;
-        if (lane == 0 && total) b = atomicAdd(mode ? c.bufc : c.outc, (unsigned long long)total);
-        b = __shfl_sync(kFull, b, 0);
-        if (lane < NW) s_base[mode][lane] = b + (incl - x);
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+      }
+      const unsigned total = __shfl_sync(kFull, incl, 31);  // per-field sums < 2^16 (NW x kCap)
+      unsigned long long b = 0;
+      if (lane == 0 && (total & 0xffffu)) b = atomicAdd(c.outc, (unsigned long long)(total & 0xffffu));
+      if (lane == 1 && (total >> 16)) b = atomicAdd(c.bufc, (unsigned long long)(total >> 16));
+      const unsigned long long br = __shfl_sync(kFull, b, 0), bcb = __shfl_sync(kFull, b, 1);
+      const unsigned ex = incl - x;
+      if (lane < NW) {
+        s_base[0][lane] = br + (ex & 0xffffu);
+        s_base[1][lane] = bcb + (ex >> 16);
       }
     }
     __syncthreads();
-    if (ocnt) wq_write<KIND, IdxT>(c.oq, ocnt, s_base[0][tid >> 5], c.kk, c.ov, c.oi, 0, sel_min, c.err);
-    if (bcnt) wq_write<KIND, IdxT>(c.bq, bcnt, s_base[1][tid >> 5], c.capa, c.bco, c.bio, 1, sel_min, c.err);
+    if (qcnt)
+      wq_write<KIND, IdxT>(wq, qcnt, s_base[0][warp], s_base[1][warp], c.ov, c.oi, c.kk, c.bco, c.bio, c.capa,
+                           sel_min, c.err);
   }
   if constexpr (DF == 3) {  // one atomic per warp: window-member extremes (the tail skips digits
                             // on which all members agree)

@@ -1,9 +1,10 @@
 // tma.cuh — Blackwell bulk-copy (TMA engine, cp.async.bulk) + mbarrier primitives (inline PTX).
 //
-// Used by the streaming passes to keep 64+ KiB per SM of the input in flight independently of the
-// registers the per-element classification needs: each warp owns a small ring of shared-memory
-// stages; lane 0 launches a 1-D bulk copy global -> shared per stage, completion is signalled on the
-// stage's mbarrier through the transaction count, and the warp consumes the stage with LDS.128.
+// Used by the streaming passes to keep ~190 KiB per SM of the input in flight independently of the
+// registers the per-element classification needs: a per-CTA ring of shared-memory stages; one
+// thread launches a 1-D bulk copy global -> shared per stage, completion is signalled on the stage's
+// "full" mbarrier through the transaction count, the warps consume the stage with LDS.128 and
+// release it on its "empty" mbarrier.
 #pragma once
 
 #include <cstdint>
@@ -27,6 +28,10 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 
 __device__ __forceinline__ void mbar_arrive_expect_tx(unsigned bar, unsigned bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive(unsigned bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
 
 // 1-D bulk copy global -> shared (this CTA), completion counted on `bar` (complete_tx::bytes).

@@ -18,10 +18,11 @@ ap.add_argument("--config", default="c3")
 ap.add_argument("--reps", type=int, default=2)
 ap.add_argument("--alpha", type=int, default=0)
 ap.add_argument("--window", type=int, default=0)
+ap.add_argument("--tma", type=int, default=0)
 a = ap.parse_args()
 c = bench.CFG[a.config]
 x = torch.from_numpy(bench.host_keys(a.config, c["n"], c["batch"])).cuda()
 for _ in range(a.reps):
-    v, i = at.select(x, c["k"], alpha=a.alpha, window=a.window)
+    v, i = at.select(x, c["k"], alpha=a.alpha, window=a.window, tma=a.tma)
 torch.cuda.synchronize()
 print("done", a.config, v.shape)
