@@ -4,6 +4,8 @@
 #include "engine_cluster.cuh"
 #include "engine_grid.cuh"
 
+#include <cstdlib>
+
 namespace airtopk {
 
 extern template cudaError_t launch_grid_kind<K_F32>(const SelectArgs&, const Plan&, const GridParams&, void*, cudaStream_t);
@@ -61,6 +63,12 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t
   gp.trace = a.trace;
   gp.samp = base + pl.off_samp;
   gp.nsms = num_sms();
+  {
+    static const char* env = getenv("AIRTOPK_BUF_PER_CTA");  // A/B knob (0 = every CTA works)
+    gp.buf_per_cta = env ? atoi(env) : kBufPerCTA;
+    static const char* env2 = getenv("AIRTOPK_SMALL_FINISH");  // A/B knob (0 = off)
+    gp.small_finish = env2 ? std::min(atoi(env2), kSmallFinish) : kSmallFinish;
+  }
   switch (a.kind) {
     case K_F32: return launch_grid_kind<K_F32>(a, pl, gp, ws, s);
     case K_F16: return launch_grid_kind<K_F16>(a, pl, gp, ws, s);

@@ -64,9 +64,92 @@ struct GridParams {
   int64_t* trace;
   void* samp;  // sample-guided window: [batch][nsamp] sampled codes
   int nsms;    // SMs of the device
+  int small_finish;  // a buffer-source pass over <= this many entries finishes the row in one CTA
+  int buf_per_cta;  // buffer-source passes: CTAs beyond ceil(nbuf / buf_per_cta) exit at once (0: all work)
 };
 
 constexpr int kBlock = 512;
+constexpr int kBufPerCTA = 0;  // buffer entries per working CTA of a buffer-source pass (0: all; measured: fewer CTAs are slower)
+constexpr int kSmallFinish = 1024;  // max buffer entries of the single-CTA finish (shared memory)
+
+// Single-CTA finish of a row: pass q reads a buffer of n <= kSmallFinish
+// entries, all sharing the prefix of digits < q-1. Its filter of digit q-1 (Alg1 L15-22) emits the
+// entries below the target digit j; among the C entries with digit q-1 == j the K smallest composite
+// keys (code, index) — the lowest-index rule of reading 1 — are the rest of the result. With C small
+// these are found by rank counting in shared memory instead of the remaining radix passes
+// (rank(e) = #{e' : (code', idx') < (code, idx)}; keys are unique, so exactly K ranks are < K).
+// Every later launch of the row returns at once (stop1 = q).
+template <int KIND, typename IdxT, int BLOCK>
+__device__ void small_finish(const PassCtx<typename KT<KIND>::U, IdxT>& c, RowState* st, unsigned char* smem) {
+  using U = typename KT<KIND>::U;
+  using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
+  __shared__ unsigned s_m;
+  U* sc = (U*)smem;
+  IdxT* si = (IdxT*)(smem + kSmallFinish * sizeof(U));
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int n = (int)c.nbuf;
+  const Digit df = c.df;
+  const unsigned long long jprev = (df.is_idx ? c.tidx : c.tcode) >> df.shift & ((1ull << df.width) - 1ull);
+  const unsigned long long Kr = st->K;
+  if (tid == 0) s_m = 0;
+  __syncthreads();
+  auto emit = [&](bool pred, U code, IdxT idx) {  // warp-aggregated result append
+    const unsigned m = __ballot_sync(kFull, pred);
+    if (!m) return;
+    unsigned long long b = 0;
+    if (lane == 0) b = atomicAdd(c.outc, (unsigned long long)__popc(m));
+    b = __shfl_sync(kFull, b, 0);
+    if (pred) {
+      const unsigned long long pos = b + __popc(m & lanemask_lt());
+      if (pos < c.kk) {
+        c.ov[pos] = from_code<KIND>(code, c.sel_min);
+        c.oi[pos] = (int64_t)idx;
+      } else {
+        atomicOr(c.err, 1u);
+      }
+    }
+  };
+  for (int b0 = 0; b0 < n; b0 += BLOCK) {
+    const int i = b0 + tid;
+    const bool valid = i < n;
+    const U code = valid ? c.bcin[i] : (U)0;
+    const IdxT idx = valid ? c.biin[i] : (IdxT)0;
+    const unsigned long long d = (df.is_idx ? (unsigned long long)idx : (unsigned long long)(W)code) >> df.shift &
+                                 ((1ull << df.width) - 1ull);
+    emit(valid && d < jprev, code, idx);
+    const bool eq = valid && d == jprev;
+    const unsigned m = __ballot_sync(kFull, eq);
+    unsigned b = 0;
+    if (lane == 0 && m) b = atomicAdd(&s_m, (unsigned)__popc(m));
+    b = __shfl_sync(kFull, b, 0);
+    if (eq) {
+      const unsigned pos = b + __popc(m & lanemask_lt());
+      sc[pos] = code;
+      si[pos] = idx;
+    }
+  }
+  __syncthreads();
+  const int m = (int)s_m;
+  for (int b0 = 0; b0 < m; b0 += BLOCK) {
+    const int i = b0 + tid;
+    bool sel = false;
+    U code = 0;
+    IdxT idx = 0;
+    if (i < m) {
+      code = sc[i];
+      idx = si[i];
+      unsigned long long rank = 0;
+      if ((unsigned long long)m > Kr)
+        for (int t = 0; t < m; ++t) rank += (sc[t] < code) || (sc[t] == code && si[t] < idx);
+      sel = rank < Kr;
+    }
+    emit(sel, code, idx);
+  }
+  if (tid == 0) {
+    if ((unsigned long long)m < Kr) atomicOr(c.err, 4u);
+    st->stop1 = c.q;  // later launches (q' > q) return at once
+  }
+}
 constexpr int kWarps = kBlock / 32;
 
 #ifndef AIRTOPK_MINB
@@ -105,6 +188,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   // ---- row state after scan q-1 ----
   const int stop1 = FILTER ? st->stop1 : 0;
   if (FILTER && stop1 != 0 && stop1 - 1 < q - 1) return;  // finished by an earlier early stop
+  if (FILTER && q < st->npass) return;                     // digit done by the window pass (digit skip)
   const int win_state = (DF == 3 || (DF == 0 && redo)) ? st->win_state : 0;
   if (DF == 3 && win_state != 1) return;                   // no window: pass 0 will read L
   if (DF == 0 && redo && win_state == 1) return;           // pass 0 was done by the window pass
@@ -121,7 +205,20 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   else c.store = c.do_hist && FILTER && (Cprev <= (unsigned long long)p.cap_rule);  // Alg1 L17
   c.sel_min = p.sel_min != 0;
   c.reverse = (q & 1) != 0;  // walk back over what the previous pass left in L2
-  c.dh = digit_of(q, KT<KIND>::R, p.IB);
+  // Window digit skip: every window member lies in [lo, hi], so the leading key digits on which lo
+  // and hi agree are common to all members (their histograms would be single bins). The window pass
+  // histograms the first digit where they may differ (qs); launches 1..qs then have nothing to do.
+  int qs = q;
+  if (DF == 3) {
+    const int pc = code_passes(KT<KIND>::R);
+    qs = 0;
+    while (qs < pc - 1) {
+      const Digit d = digit_of(qs, KT<KIND>::R, p.IB);
+      if ((st->win_lo >> d.shift) != (st->win_hi >> d.shift)) break;
+      ++qs;
+    }
+  }
+  c.dh = digit_of(qs, KT<KIND>::R, p.IB);
   c.df = digit_of(FILTER ? q - 1 : 0, KT<KIND>::R, p.IB);
   c.tcode = FILTER ? st->tcode : 0ull;
   c.tidx = FILTER ? st->tidx : 0ull;
@@ -132,8 +229,16 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.rowp = (const U*)p.keys + row * p.len;
   c.rowi = HASIDX ? p.in_idx + row * p.len : nullptr;
   c.len = p.len;
+  // A pass over a (small) candidate buffer needs few CTAs: only the first `act` take part (fewer
+  // same-address histogram merges and ticket arrivals); the others leave right away.
+  int act = p.cpr;
+  if (src1 > 0 && p.buf_per_cta > 0) {
+    const unsigned long long nb = st->buf_count[src1 - 1];
+    act = (int)min((unsigned long long)p.cpr, max(1ull, (nb + p.buf_per_cta - 1) / (unsigned long long)p.buf_per_cta));
+    if (cta >= act) return;
+  }
   c.slice = cta;
-  c.nslices = p.cpr;
+  c.nslices = act;
   const int islot = src1 > 0 ? src1 - 1 : 0;
   c.bcin = (const U*)p.bcode + ((size_t)islot * p.batch + row) * p.cap_alloc;
   c.biin = (const IdxT*)p.bidx + ((size_t)islot * p.batch + row) * p.cap_alloc;
@@ -151,6 +256,12 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.ring = smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>();
   c.wq = &sh_wq[HAS_Q ? warp : 0];
 
+  if constexpr (FILTER && DH != 0) {
+    if (!c.emit_all && !c.srcL && c.nbuf <= (unsigned long long)p.small_finish && p.trace == nullptr) {
+      if (cta == 0) small_finish<KIND, IdxT, kBlock>(c, st, (unsigned char*)sh_hist);
+      return;
+    }
+  }
   const bool hist_on = c.do_hist || DF == 0 || DF == 3;
   if (hist_on) {
     for (int i = tid; i < kHistSlots * HC; i += kBlock) sh_hist[i] = 0;
@@ -173,7 +284,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
     if (v) atomicAdd(&gh[i], (CountT)v);
   }
   __syncthreads();  // the CTA's histogram merge / queue flushes precede thread 0's release
-  if (tid == 0) sh_last = (ticket_arrive(&st->ticket) == (unsigned)(p.cpr - 1));
+  if (tid == 0) sh_last = (ticket_arrive(&st->ticket) == (unsigned)(act - 1));
   __syncthreads();
   if (!sh_last) return;
 
@@ -203,7 +314,8 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   }
   const ScanResult r = scan_choose<kBlock>(
       [&](int b) { return (unsigned long long)__ldcg(&gh[b]); }, nb, Kin, sh_tmp, &sh_res);
-  CountT* gh2 = (CountT*)p.ghist + ((size_t)row * 2 + ((q + 1) & 1)) * kMaxBins;
+  __syncthreads();  // (after a window digit skip the next pass may use the slot just scanned)
+  CountT* gh2 = (CountT*)p.ghist + ((size_t)row * 2 + ((qs + 1) & 1)) * kMaxBins;
   for (int i = tid; i < kMaxBins; i += kBlock) gh2[i] = 0;
   if (tid == 0) {
     int next_src1 = (c.store) ? sslot + 1 : src1;  // the buffer this pass wrote feeds the next one
@@ -213,10 +325,11 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
       st->Cp = Cin;
       st->C = newC;
       st->K = newK;
+      if (DF == 3 && qs > 0) st->tcode = st->win_lo >> (dh.shift + dh.width) << (dh.shift + dh.width);
       if (!dh.is_idx) st->tcode |= (unsigned long long)r.j << dh.shift;
       else st->tidx |= (unsigned long long)r.j << dh.shift;
       st->j = r.j;
-      st->npass = q + 1;
+      st->npass = qs + 1;
       if (newK == newC) st->stop1 = q + 1;                             // early stop
       st->src1 = next_src1;
       st->buf_count[next_src1 == 1 ? 1 : 0] = 0;                        // next pass's output buffer
@@ -585,6 +698,8 @@ struct Events {
 
 template <int KIND, typename IdxT, int DF, int DH, bool TMA = false>
 constexpr size_t hist_smem_bytes() {
+  static_assert(!(DF == 1 || DF == 2) || DH == 0 || (size_t)kHistSlots * 4 * hist_copies<KIND, IdxT, DF>() >=
+                    (size_t)kSmallFinish * (sizeof(typename KT<KIND>::U) + sizeof(IdxT)), "small finish smem");
   constexpr int HC = hist_copies<KIND, IdxT, DF>();
   return TMA ? tma_smem_bytes<HC>() : (size_t)kHistSlots * 4 * HC;
 }

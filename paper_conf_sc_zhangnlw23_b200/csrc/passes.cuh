@@ -314,7 +314,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
       if (cd) {  // window member: extremes + the pass-1 digit histogram of the window buffer
         wlo_seen = ((W)code < wlo_seen) ? (W)code : wlo_seen;
         whi_seen = ((W)code > whi_seen) ? (W)code : whi_seen;
-        shared_inc(hbase + 4u * (unsigned)((W)code >> shh));
+        shared_inc(hbase + 4u * (unsigned)(((W)code >> shh) & hmask));
       }
     }
     return w ? 0 : ((cd && store) ? 1 : 2);

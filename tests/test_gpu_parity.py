@@ -345,3 +345,46 @@ def test_tma_streaming(tma, window, dist, m, batch, n, k, off):
     for sm in (True, False):
         v, i = gpu_select(x, "f32", k, sm, offset_elems=off, tma=tma, window=window, engine=1)
         assert_parity(x, "f32", k, sm, v, i)
+
+
+# ---------------------------------------------------------------- rows longer than 2^32 (64-bit indices)
+
+@pytest.mark.parametrize("dtn,largest", [("f16", False), ("f32", False), ("f16", True)])
+def test_row_longer_than_2p32(dtn, largest):
+    """len = 2^32 + 2^20 + 3 (the u64-index path, include/airtopk.h "Limits"; the c5 row
+    on one GPU). Every key equals v0 except planted keys at positions on both sides of 2^32, some
+    equal to each other and some equal to v0's neighbours. Property that holds at any size: the
+    top-K of such a row = the top-K of the sub-row made of the planted positions plus the K lowest
+    non-planted positions (all v0), kept in index order, since every other element is a v0 with a
+    higher index (P:78 with the lowest-index rule). That sub-row goes to the CPU oracle."""
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    n = (1 << 32) + (1 << 20) + 3
+    k = 97
+    npdt = {"f16": np.float16, "f32": np.float32}[dtn]
+    tdt = {"f16": torch.float16, "f32": torch.float32}[dtn]
+    rng = np.random.default_rng(4321)
+    pos = np.unique(np.concatenate([
+        rng.integers(0, 1 << 32, 40), rng.integers(1 << 32, n, 40),
+        [0, 5, (1 << 32) - 1, 1 << 32, (1 << 32) + 1, n - 1]]).astype(np.int64))
+    vals = rng.choice(np.array([0.25, 0.5, 0.75, 1.0, 1.5, 2.0, -3.0, 7.0], dtype=npdt), pos.size)
+    v0 = npdt(1.0)
+    x = torch.full((n,), float(v0), dtype=tdt, device="cuda")
+    x[torch.from_numpy(pos).cuda()] = torch.from_numpy(vals).cuda()
+    v, i = at.select(x.reshape(1, n), k, largest=largest)
+    torch.cuda.synchronize()
+    # the sub-row: planted positions + the k lowest positions holding v0 that were not planted
+    fill = np.setdiff1d(np.arange(k + pos.size, dtype=np.int64), pos)[:k]
+    sub_pos = np.concatenate([pos, fill])
+    order = np.argsort(sub_pos)
+    sub_pos = sub_pos[order]
+    sub_val = np.concatenate([vals, np.full(fill.size, v0, npdt)])[order]
+    bits = {"f16": np.uint16, "f32": np.uint32}[dtn]
+    rv, ri = oracle.topk_nth(sub_val.view(bits)[None, :], k, not largest, dt=oracle.DT_NAMES[dtn])
+    gi = np.sort(i.cpu().numpy()[0])
+    assert gi.max() >= 0
+    assert np.array_equal(gi, np.sort(sub_pos[ri[0]])), "index set differs (64-bit index path)"
+    gv = to_bits(v, dtn)[0]
+    assert np.array_equal(np.sort(gv), np.sort(rv[0].view(bits)))
+    del x
+    torch.cuda.empty_cache()
