@@ -41,8 +41,10 @@ CFG = {
     "c2": dict(batch=100, n=1 << 20, k=256, dist="normal"),
     "c3": dict(batch=1, n=1 << 30, k=1 << 20, dist="uniform"),
     "c4": dict(batch=1, n=1 << 28, k=50000, dist="adversarial"),
+    # one 2^33 row: on one GPU the whole row (64-bit index path), at N ranks a 2^33/N shard each
+    "c5": dict(batch=1, n=1 << 33, k=1 << 16, dist="uniform"),
 }
-DEFAULT_STEPS = {"c1": 200, "c2": 100, "c3": 60, "c4": 60}
+DEFAULT_STEPS = {"c1": 200, "c2": 100, "c3": 60, "c4": 60, "c5": 10}
 
 
 def log(*a):
@@ -217,7 +219,13 @@ def main():
     peak, peak_kind = hbm_peak()
 
     # ---------------- workload on this rank
-    if cfg == "c2":
+    if cfg == "c5":  # the fixed 2^33 row split across the ranks (total work fixed -> "strong")
+        batch, n = 1, c["n"] // world
+        xh = host_keys(cfg, n, 1, offset=rank * n)
+        scaling = "strong"
+        total_units = c["n"]
+        split = world > 1
+    elif cfg == "c2":
         lo, hi = atdist.row_range(c["batch"], rank, world)
         batch, n = hi - lo, c["n"]
         xh = host_keys(cfg, n, batch, offset=lo * n)

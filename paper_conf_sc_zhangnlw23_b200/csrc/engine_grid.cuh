@@ -162,6 +162,20 @@ constexpr int kMinBlocksFilter = AIRTOPK_SLOW_REG ? 2 : AIRTOPK_MINB;
 // sample-guided window pass (q = 0); `redo` = the pass-0 histogram re-run over the window buffer.
 // TMA: the input row is streamed through per-warp shared rings by the bulk-copy engine (1 CTA/SM,
 // DESIGN.md "Kernels"); otherwise 4 x 16-byte register loads per thread (3 CTAs/SM).
+// Debug timing of pass q (trace mode only; trace slot 7 + q of the row, zero-initialised):
+// [0] ~min CTA start, [1] max run_pass end, [2] max ticket arrival, [3] last CTA: scan done,
+// [4] CTA 0 start, [5] CTA 0 run_pass end
+__device__ __forceinline__ void dbg_stamp(int64_t* trace, int64_t row, int q, int f, int mode, int P) {
+  // only slots no pass record uses (passes 0..P fill slots 0..P; slot 15: sample_kernel)
+  if (trace == nullptr || threadIdx.x != 0 || 7 + q >= kTraceMaxPasses - 1 || 7 + q <= P) return;
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  unsigned long long* a = (unsigned long long*)(trace + ((size_t)row * kTraceMaxPasses + 7 + q) * kTraceFields + f);
+  if (mode == 0) atomicMax(a, ~t);
+  else if (mode == 1) atomicMax(a, t);
+  else *a = t;
+}
+
 template <int KIND, typename IdxT, int DF, int DH, bool HASIDX, bool TMA = false>
 __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMinBlocksFilter))
     pass_kernel(const GridParams p, const int q, const int redo) {
@@ -262,6 +276,8 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
       return;
     }
   }
+  dbg_stamp(p.trace, row, q, 0, 0, p.P);
+  if (cta == 0) dbg_stamp(p.trace, row, q, 4, 2, p.P);
   const bool hist_on = c.do_hist || DF == 0 || DF == 3;
   if (hist_on) {
     for (int i = tid; i < kHistSlots * HC; i += kBlock) sh_hist[i] = 0;
@@ -269,6 +285,8 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   }
 
   const unsigned long long nread = run_pass<KIND, IdxT, DF, DH, HASIDX, kBlock, 0, TMA>(c);
+  dbg_stamp(p.trace, row, q, 1, 1, p.P);
+  if (cta == 0) dbg_stamp(p.trace, row, q, 5, 2, p.P);
 
   if (!hist_on) return;
 
@@ -284,6 +302,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
     if (v) atomicAdd(&gh[i], (CountT)v);
   }
   __syncthreads();  // the CTA's histogram merge / queue flushes precede thread 0's release
+  dbg_stamp(p.trace, row, q, 2, 1, p.P);
   if (tid == 0) sh_last = (ticket_arrive(&st->ticket) == (unsigned)(act - 1));
   __syncthreads();
   if (!sh_last) return;
@@ -342,6 +361,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
     }
     st->ticket = 0;
   }
+  dbg_stamp(p.trace, row, q, 3, 2, p.P);
 }
 
 // Sample-guided window: one CTA per row reads S
@@ -567,38 +587,44 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
   const int nruns = nsamp / kRun;
   const int64_t stride = p.len / nruns;
   // phase 1: this CTA's runs part, part + cps, ... (all loads in flight at once)
+  constexpr int PER = kMaxSamples / kSampleBlock;
+  W v[PER];  // phase 2: sample t * kSampleBlock + tid (valid for t < tv)
   {
-    constexpr int PER = kMaxSamples / kSampleBlock;
     const int runs_here = (nruns - part + cps - 1) / cps;  // runs part, part + cps, ...
     const int tmax = (runs_here * kRun + kSampleBlock - 1) / kSampleBlock;
-    U v[PER];
+    U x[PER];
 #pragma unroll
     for (int t = 0; t < PER; ++t) {
       const int slot = t * kSampleBlock + threadIdx.x;  // (run-in-part, lane)
       const int run = (slot / kRun) * cps + part, e = slot % kRun;
       const int64_t pos = (int64_t)run * stride + (stride - kRun) / 2 + e;
-      if (t < tmax && run < nruns && pos < p.len) v[t] = __ldg(rowp + pos);
+      if (t < tmax && run < nruns && pos < p.len) x[t] = __ldg(rowp + pos);
     }
 #pragma unroll
     for (int t = 0; t < PER; ++t) {
       const int slot = t * kSampleBlock + threadIdx.x;
       const int run = (slot / kRun) * cps + part, e = slot % kRun;
       const int64_t pos = (int64_t)run * stride + (stride - kRun) / 2 + e;
-      if (t < tmax && run < nruns && pos < p.len) samp[run * kRun + e] = (W)to_code_x<KIND>(v[t], xmask);
+      const bool ok = t < tmax && run < nruns && pos < p.len;
+      const W code = ok ? (W)to_code_x<KIND>(x[t], xmask) : (W)0;
+      if (cps == 1) v[t] = code;  // one CTA per row: sample slot == run * kRun + e, kept in registers
+      else if (ok) samp[run * kRun + e] = code;
     }
   }
-  __syncthreads();
-  if (threadIdx.x == 0) sh_last = (ticket_arrive(&st->ticket) == (unsigned)(cps - 1));
-  __syncthreads();
-  if (!sh_last) return;
+  if (cps > 1) {
+    __syncthreads();
+    if (threadIdx.x == 0) sh_last = (ticket_arrive(&st->ticket) == (unsigned)(cps - 1));
+    __syncthreads();
+    if (!sh_last) return;
+  }
   stamp(2);
   // phase 2 (last CTA of the row): the window from the sample order statistics; the samples stay
   // in registers (16 per thread)
-  constexpr int PER = kMaxSamples / kSampleBlock;
   const int tv = (nsamp - (int)threadIdx.x + kSampleBlock - 1) / kSampleBlock;  // valid v[t]: t < tv
-  W v[PER];
+  if (cps > 1) {
 #pragma unroll
-  for (int t = 0; t < PER; ++t) v[t] = (t < tv) ? __ldcg(samp + t * kSampleBlock + threadIdx.x) : (W)0;
+    for (int t = 0; t < PER; ++t) v[t] = (t < tv) ? __ldcg(samp + t * kSampleBlock + threadIdx.x) : (W)0;
+  }
   {
     W lmin = ~(W)0, lmax = 0;
 #pragma unroll

@@ -18,3 +18,7 @@ timeout 600 ncu --set full --clock-control none --import-source on -k regex:pass
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:cluster_kernel -s 1 -c 1 -o gpurun_out/full_c4_tail python tools/prof_select.py --config c4 --reps 2 > gpurun_out/ncu_t.log 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:pass_kernel -s 7 -c 2 -o gpurun_out/full_c3_paper python tools/prof_select.py --config c3 --reps 2 --window -1 > gpurun_out/ncu_p.log 2>&1
 ls -la gpurun_out | tail -30
+# the first buffer pass after the window (c3) and the sample kernel, with source pages
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:pass_kernel -s 10 -c 1 -o gpurun_out/full_c3_q1 python tools/prof_select.py --config c3 --reps 2 > gpurun_out/ncu_q1.log 2>&1
+ncu -i gpurun_out/full_c3_q1.ncu-rep --page source --csv --print-source sass > gpurun_out/src_c3_q1.csv 2>/dev/null
+ncu -i gpurun_out/full_c3_window.ncu-rep --page source --csv --print-source sass > gpurun_out/src_c3_window.csv 2>/dev/null
