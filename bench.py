@@ -412,6 +412,8 @@ def launch_names(plan):
         return ["cluster_kernel (all passes)"], [True]
     if plan["engine"] == 3:
         return ["trivial_copy"], [True]
+    if plan["engine"] == 4:
+        return ["gridselect_kernel (GridSelect, P:188-204)"], [True]
     P = plan["passes"]
     L = plan["launches"]
     if L not in (P + 1, P + 3):  # window pass + tail_q grid passes + one cluster-engine tail launch

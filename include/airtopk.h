@@ -78,7 +78,13 @@ typedef enum {
 typedef enum {
   AIRTOPK_ENGINE_AUTO = 0,
   AIRTOPK_ENGINE_GRID = 1,    /* multi-CTA per row, one launch per pass, last-CTA scan */
-  AIRTOPK_ENGINE_CLUSTER = 2  /* one thread-block cluster per row, all passes in one launch */
+  AIRTOPK_ENGINE_CLUSTER = 2, /* one thread-block cluster per row, all passes in one launch */
+  AIRTOPK_ENGINE_GRIDSELECT = 4 /* the paper's second algorithm (§4): per-warp shared
+                                   32-entry queue with two-step ballot insertion, sorted per-warp
+                                   top-K lists merged by the last CTA of the row. Same results
+                                   (lowest-index ties). Only for keys of <= 32 bits, len < 2^32 and
+                                   K <= 256, else AIRTOPK_EINVAL. Rows come out sorted. Never chosen
+                                   by AUTO. */
 } airtopk_engine;
 
 /* Tuning / ablation knobs. Pass NULL for the defaults. */

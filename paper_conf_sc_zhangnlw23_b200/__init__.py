@@ -11,10 +11,10 @@ from __future__ import annotations
 import ctypes
 
 from . import _lib
-from ._lib import AirTopKError, Options, OK, ENGINE_AUTO, ENGINE_GRID, ENGINE_CLUSTER, TRACE_MAX_PASSES
+from ._lib import AirTopKError, Options, OK, ENGINE_AUTO, ENGINE_GRID, ENGINE_CLUSTER, ENGINE_GRIDSELECT, TRACE_MAX_PASSES
 
 __all__ = ["select", "select_with_idx", "select_host", "workspace_bytes", "describe", "lib", "AirTopKError",
-           "ENGINE_AUTO", "ENGINE_GRID", "ENGINE_CLUSTER", "dtype_code"]
+           "ENGINE_AUTO", "ENGINE_GRID", "ENGINE_CLUSTER", "ENGINE_GRIDSELECT", "dtype_code"]
 
 _LIB = None
 

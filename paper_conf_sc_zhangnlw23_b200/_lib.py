@@ -12,7 +12,7 @@ LIB_PATH = os.environ.get("AIRTOPK_LIB", os.path.join(_PKG, "libairtopk.so"))
 
 OK, EINVAL, EDTYPE, ENOSPACE, ECUDA = 0, 1, 2, 3, 4
 F32, F16, BF16, F64, U32 = 0, 1, 2, 3, 4
-ENGINE_AUTO, ENGINE_GRID, ENGINE_CLUSTER = 0, 1, 2
+ENGINE_AUTO, ENGINE_GRID, ENGINE_CLUSTER, ENGINE_GRIDSELECT = 0, 1, 2, 4
 TRACE_MAX_PASSES = 16
 TRACE_FIELDS = ("width", "src_L", "stored", "j", "K", "C", "Cp", "emitted", "early_stop", "read")
 

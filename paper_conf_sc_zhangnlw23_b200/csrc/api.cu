@@ -63,6 +63,12 @@ Plan make_plan(const SelectArgs& a) {
     p.engine = 3;
     return p;
   }
+  if (a.engine == 4) {  // GridSelect (the paper's second algorithm)
+    p.engine = 4;
+    p.cpr = gridselect_ctas(a);
+    p.bytes = gridselect_workspace(a, p.cpr);
+    return p;
+  }
   p.idx64 = (a.in_idx != nullptr) || (a.len > (int64_t(1) << 32));
   p.IB = a.in_idx ? a.idx_bits : bits_needed((uint64_t)(a.len - 1));
   p.P = code_passes(p.R) + idx_passes(p.IB);
@@ -112,7 +118,7 @@ static int auto_cluster_size(const SelectArgs& a) {
 constexpr double kTailPerCTA = 4096.0;  // expected window entries per cluster-tail CTA
 
 static void choose_launch(const SelectArgs& a, Plan& p) {
-  if (p.engine == 3) return;
+  if (p.engine == 3 || p.engine == 4) return;
   p.engine = a.engine > 0 ? a.engine : auto_engine(a);
   if (p.engine == 2) {
     p.csize = auto_cluster_size(a);
@@ -169,7 +175,8 @@ static airtopk_status validate(const SelectArgs& a) {
   if (!a.keys || !a.out_vals || !a.out_idx) return AIRTOPK_EINVAL;
   if (a.batch < 1 || a.len < 1 || a.k < 1 || a.k > a.len) return AIRTOPK_EINVAL;
   if (a.alpha < 0) return AIRTOPK_EINVAL;
-  if (a.engine < 0 || a.engine > 2) return AIRTOPK_EINVAL;
+  if (a.engine < 0 || a.engine > 4 || a.engine == 3) return AIRTOPK_EINVAL;
+  if (a.engine == 4 && !gridselect_supported(a)) return AIRTOPK_EINVAL;
   if (a.window < -1 || a.window > 1) return AIRTOPK_EINVAL;
   if (a.in_idx && (a.batch != 1 || a.idx_bits < 1 || a.idx_bits > 63)) return AIRTOPK_EINVAL;
   return AIRTOPK_OK;
@@ -190,6 +197,10 @@ static airtopk_status run(const SelectArgs& a, void* ws, size_t ws_bytes, cudaSt
   }
   if (!ws || ws_bytes < p.bytes) return AIRTOPK_ENOSPACE;
   if (((uintptr_t)ws & 255u) != 0) return AIRTOPK_EINVAL;
+  if (p.engine == 4) {
+    cudaError_t e = run_gridselect(a, ws, ws_bytes, s);
+    return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
+  }
   choose_launch(a, p);
   if (p.engine == 2 && (p.csize < 1 || p.csize > 16 || (p.csize & (p.csize - 1)))) return AIRTOPK_EINVAL;
   cudaError_t e = (p.engine == 2) ? run_cluster(a, p, ws, s) : run_grid(a, p, ws, s);
@@ -372,8 +383,8 @@ airtopk_status airtopk_describe(airtopk_dtype dtype, int64_t batch, int64_t len,
   std::memset(out, 0, sizeof(*out));
   out->engine = p.engine;
   out->passes = p.P;
-  out->launches = p.engine == 3 ? 1 : (p.engine == 2 ? 1 : (p.tail ? 3 + p.tail_q : p.P + 1 + (p.nsamp > 0 ? 2 : 0)));
-  out->ctas_per_row = p.engine == 1 ? p.cpr : 0;
+  out->launches = (p.engine == 3 || p.engine == 4) ? 1 : (p.engine == 2 ? 1 : (p.tail ? 3 + p.tail_q : p.P + 1 + (p.nsamp > 0 ? 2 : 0)));
+  out->ctas_per_row = (p.engine == 1 || p.engine == 4) ? p.cpr : 0;
   out->cluster_size = (p.engine == 2 || p.tail) ? p.csize : 0;
   out->index_bits = p.IB;
   out->buffer_cap = p.cap_rule;

@@ -29,7 +29,7 @@ struct SelectArgs {
 
 // Resolved launch plan (host side).
 struct Plan {
-  int engine;        // 1 grid, 2 cluster, 3 trivial copy (K == N)
+  int engine;        // 1 grid, 2 cluster, 3 trivial copy (K == N), 4 GridSelect
   int idx64;         // 64-bit internal indices
   int R;             // key bits
   int IB;            // index bits appended to the key for the lowest-index tie-break
@@ -55,5 +55,10 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t 
 cudaError_t run_cluster(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 cudaError_t run_trivial(const SelectArgs& a, cudaStream_t s);
 int grid_blocks_per_sm(const SelectArgs& a, int idx64);
+// GridSelect: keys of <= 32 bits, len < 2^32, K <= 256
+bool gridselect_supported(const SelectArgs& a);
+int gridselect_ctas(const SelectArgs& a);
+size_t gridselect_workspace(const SelectArgs& a, int G);
+cudaError_t run_gridselect(const SelectArgs& a, void* ws, size_t ws_bytes, cudaStream_t s);
 
 }  // namespace airtopk

@@ -17,6 +17,7 @@
 #pragma once
 
 #include <cooperative_groups.h>
+#include <cstdlib>
 
 #include "device.cuh"
 #include "engine.h"
@@ -45,11 +46,11 @@ struct ClusterParams {
   int nclusters;
   int tail;      // 1: continue rows after the grid engine's window pass
   int tail_q;    // tail mode: the grid engine ran passes q < tail_q after the window pass
+  int timing_stride;  // int64 slots per CTA in `timing` (8; 24 with the merge-phase stamps, debug)
   int64_t* timing;  // optional: per CTA [globaltimer at start, at end, rows done, passes run, end of passes 1-4]
 };
 
 struct ClusterShared {
-  unsigned long long segtot[kMaxCluster];  // segment totals, written remotely by each CTA
   unsigned long long res_before, res_cnt;  // target digit result, written remotely by the owner
   unsigned res_j;
   unsigned long long tmp[kCWarps];
@@ -72,7 +73,7 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
   extern __shared__ unsigned sh_hist[];  // kHistSlots counters
   __shared__ WarpQ<U, IdxT> sh_wq[kCWarps];
   __shared__ ClusterShared cs;
-  __shared__ unsigned sh_seg[kMaxBins];  // this CTA's merged bin segment
+  __shared__ unsigned sh_seg[kMaxBins];  // the cluster's merged histogram (each CTA's copy)
 
   cg::cluster_group cl = cg::this_cluster();
   const int CS = (int)cl.num_blocks();
@@ -88,6 +89,14 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
   unsigned long long t_start = 0;
   int n_rows = 0, n_passes = 0;
   if (p.timing && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
+  // debug timing of the merge / scan phases of the first two passes (slots 8 + 5 * pass + phase)
+  auto stamp = [&](int phase) {
+    if (p.timing && p.timing_stride >= 24 && tid == 0 && n_passes >= 1 && n_passes <= 2) {
+      unsigned long long tp;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tp));
+      p.timing[(int64_t)blockIdx.x * p.timing_stride + 8 + 5 * (n_passes - 1) + phase] = (int64_t)tp;
+    }
+  };
 
   for (int64_t row = cid; row < p.batch; row += p.nclusters) {
     RowState* st = p.st + row;
@@ -95,6 +104,15 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
     int stop1 = 0, src1 = 0;  // src1: 0 = the input row L, s + 1 = candidate buffer slot s
     int q0 = 0;
     const int ws = p.tail ? st->win_state : 0;
+    if (!p.tail) {  // standalone: the row's counters start at zero (no memset launch before the kernel)
+      if (crank == 0 && tid == 0) {
+        st->out_count = 0;
+        st->buf_count[0] = 0;
+        st->buf_count[1] = 0;
+        st->error = 0;
+      }
+      cl.sync();
+    }
     if (p.tail && (ws == 1 || p.tail_q > 0)) {
       // continue the row from its state: after the window pass (which scanned pass 1 over the window
       // buffer) or after the grid passes q < tail_q
@@ -179,7 +197,7 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
       if (p.timing && tid == 0 && n_passes <= 4) {
         unsigned long long tp;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tp));
-        p.timing[(int64_t)blockIdx.x * 8 + 3 + n_passes] = (int64_t)tp;
+        p.timing[(int64_t)blockIdx.x * p.timing_stride + 3 + n_passes] = (int64_t)tp;
       }
       if (!hist_on) break;  // emit-all pass: the row is complete
 
@@ -200,50 +218,39 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
         __syncthreads();
       } else {
         cl.sync();  // (B) every CTA's histogram and appends are complete
-        // CTA r owns bins [r*seg, (r+1)*seg): sum them over the cluster (all DSMEM loads in flight)
+        stamp(0);
+        // CTA r owns bins [r*seg, (r+1)*seg): sums them over the cluster (all CS DSMEM loads of a bin
+        // in flight at once) and stores the sums into EVERY CTA's full merged histogram (sh_seg), so
+        // that after the next barrier each CTA scans all bins locally (no remote loads on the scan)
         const int seg = (nb + CS - 1) / CS;
         const int b0 = crank * seg;
-        for (int i = tid; i < seg; i += kCBlock) sh_seg[i] = 0;
-        __syncthreads();
-        const int pairs = seg * CS;
-        for (int pr = tid; pr < pairs; pr += kCBlock) {
-          const int b = pr % seg, rr = pr / seg;
-          const unsigned v = (b0 + b < nb) ? cl.map_shared_rank(sh_hist, rr)[b0 + b] : 0u;
-          if (v) atomicAdd(&sh_seg[b], v);
-        }
-        __syncthreads();
-        unsigned long long mytot = 0;
-        for (int i = tid; i < seg; i += kCBlock) mytot += sh_seg[i];
-        {
-          unsigned long long tot;
-          (void)block_exclusive_scan<kCBlock>(mytot, cs.tmp, tot);
-          if (tid < CS) cl.map_shared_rank(&cs, tid)->segtot[crank] = tot;
-        }
-        if (c.store) src1 = sslot + 1;
-        if (crank == 0 && tid == 0) st->buf_count[src1 == 1 ? 1 : 0] = 0;  // next pass's output buffer
-        cl.sync();  // (C) segment totals published; remote reads of sh_hist done
-        // every CTA finds the owner segment and scans the owner's merged bins (DSMEM) itself:
-        // identical result everywhere, no broadcast barrier
-        unsigned long long before_seg = 0;
-        int owner = 0;
-        {
-          unsigned long long run = 0;
-          bool found = false;
-          for (int rr = 0; rr < CS; ++rr) {
-            const unsigned long long t = cs.segtot[rr];
-            if (!found && run < K && run + t >= K) { owner = rr; before_seg = run; found = true; }
-            run += t;
+        for (int b = tid; b < seg; b += kCBlock) {
+          if (b0 + b < nb) {
+            unsigned x[kMaxCluster];
+#pragma unroll
+            for (int rr = 0; rr < kMaxCluster; ++rr) x[rr] = (rr < CS) ? cl.map_shared_rank(sh_hist, rr)[b0 + b] : 0u;
+            unsigned v = 0;
+#pragma unroll
+            for (int rr = 0; rr < kMaxCluster; ++rr) v += x[rr];
+#pragma unroll
+            for (int rr = 0; rr < kMaxCluster; ++rr)
+              if (rr < CS) cl.map_shared_rank(sh_seg, rr)[b0 + b] = v;
           }
         }
-        const unsigned* oseg = cl.map_shared_rank(sh_seg, owner);
+        stamp(1);
+        if (c.store) src1 = sslot + 1;
+        if (crank == 0 && tid == 0) st->buf_count[src1 == 1 ? 1 : 0] = 0;  // next pass's output buffer
+        cl.sync();  // (C) merged histogram complete everywhere; remote reads of sh_hist done
+        stamp(2);
         const ScanResult r = scan_choose<kCBlock>(
-            [&](int b) { return (unsigned long long)oseg[b]; }, seg, K - before_seg, cs.tmp, &cs.scan);
+            [&](int b) { return (unsigned long long)sh_seg[b]; }, nb, K, cs.tmp, &cs.scan);
         if (tid == 0) {
-          cs.res_j = (unsigned)(owner * seg + r.j);
-          cs.res_before = before_seg + r.before;
+          cs.res_j = r.j;
+          cs.res_before = r.before;
           cs.res_cnt = r.cnt;
         }
         __syncthreads();
+        stamp(3);
       }
       const unsigned j = cs.res_j;
       const unsigned long long newK = K - cs.res_before, newC = cs.res_cnt;   // Alg1 L26-28
@@ -260,7 +267,7 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
   if (p.timing && tid == 0) {
     unsigned long long t_end;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
-    int64_t* t = p.timing + (int64_t)blockIdx.x * 8;
+    int64_t* t = p.timing + (int64_t)blockIdx.x * p.timing_stride;
     t[0] = (int64_t)t_start; t[1] = (int64_t)t_end; t[2] = n_rows; t[3] = n_passes;
   }
 }
@@ -279,10 +286,6 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   if (attr2 != cudaSuccess) return attr2;
   char* base = (char*)ws;
   cudaError_t e = cudaSuccess;
-  if (!tail) {  // standalone: fresh row states (the tail mode continues the grid engine's)
-    e = cudaMemsetAsync(base + pl.off_state, 0, pl.off_hist - pl.off_state, s);
-    if (e != cudaSuccess) return e;
-  }
   ClusterParams p;
   p.keys = a.keys;
   p.in_idx = a.in_idx;
@@ -302,6 +305,7 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   p.tail = tail;
   p.tail_q = pl.tail_q;
   p.timing = a.trace;  // cluster engine: the trace buffer receives per-CTA timing instead
+  p.timing_stride = getenv("AIRTOPK_CLUSTER_TIMING") ? 24 : 8;
 
   cudaLaunchConfig_t cfg = {};
   cudaLaunchAttribute at[2];

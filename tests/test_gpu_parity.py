@@ -388,3 +388,37 @@ def test_row_longer_than_2p32(dtn, largest):
     assert np.array_equal(np.sort(gv), np.sort(rv[0].view(bits)))
     del x
     torch.cuda.empty_cache()
+
+
+# ---------------------------------------------------------------- GridSelect (NEXT #3)
+
+@pytest.mark.parametrize("dist,m", [("uniform", 20), ("normal", 20), ("adversarial", 20), ("adversarial", 28)])
+@pytest.mark.parametrize("batch,n,k", [(1, 1 << 16, 32), (1, 1 << 16, 1), (3, 100003, 256), (5, 1000, 100),
+                                       (2, 33, 33), (4, 31, 7), (1, 1 << 20, 200)])
+@pytest.mark.parametrize("select_min", [True, False])
+def test_gridselect(dist, m, batch, n, k, select_min):
+    x = _keys(dist, 131, batch, n, m=m)
+    v, i = gpu_select(x, "f32", k, select_min, engine=4)
+    assert_parity(x, "f32", k, select_min, v, i)
+
+
+@pytest.mark.parametrize("dtn", ["f16", "bf16", "u32"])
+def test_gridselect_dtypes(dtn):
+    u = gen.u64(92, 6 * 20011)
+    raw = u.astype({"f16": np.uint16, "bf16": np.uint16, "u32": np.uint32}[dtn]).reshape(6, 20011)
+    for k in (1, 64, 256):
+        for sm in (True, False):
+            v, i = gpu_select(raw, dtn, k, sm, engine=4)
+            assert_parity(raw, dtn, k, sm, v, i)
+
+
+def test_gridselect_sorted_output_and_c1():
+    """GridSelect returns each row sorted in the selection order (composite key, lowest index first
+    among equal keys), on the c1 workload."""
+    x = gen.config_keys("c1")
+    v, i = gpu_select(x, "f32", 32, True, engine=4)
+    assert_parity(x, "f32", 32, True, v, i)
+    vals = v.reshape(-1).view(np.float32).astype(np.float64)
+    idx = i.reshape(-1)
+    for a in range(31):
+        assert vals[a] < vals[a + 1] or (vals[a] == vals[a + 1] and idx[a] < idx[a + 1])
