@@ -196,6 +196,13 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
   RowState* st = p.st + row;
+  // Window pass over bulk-copy rings: the ring's first stages depend only on the (read-only) keys, so
+  // they are issued before pdl_wait and fill while the sample kernel finishes.
+  int pre = 0;
+  if constexpr (DF == 3 && TMA)
+    pre = tma_prologue<typename KT<KIND>::U, hist_copies<KIND, IdxT, DF>(), kBlock>(
+        (const typename KT<KIND>::U*)p.keys + row * p.len, p.len, cta, p.cpr, false,
+        smem_addr(sh_hist) + (unsigned)tma_ring_offset<hist_copies<KIND, IdxT, DF>()>());
   pdl_wait();     // the previous pass's scan (row state, buffers) is complete and visible
   pdl_trigger();  // the next pass may be scheduled as our CTAs retire (hides launch latency)
 
@@ -204,7 +211,14 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   if (FILTER && stop1 != 0 && stop1 - 1 < q - 1) return;  // finished by an earlier early stop
   if (FILTER && q < st->npass) return;                     // digit done by the window pass (digit skip)
   const int win_state = (DF == 3 || (DF == 0 && redo)) ? st->win_state : 0;
-  if (DF == 3 && win_state != 1) return;                   // no window: pass 0 will read L
+  if (DF == 3 && win_state != 1) {                         // no window: pass 0 will read L
+    if constexpr (DF == 3 && TMA) {  // (thread 0) the pre-issued copies must land before the CTA exits
+      const unsigned fullb = smem_addr(sh_hist) + (unsigned)tma_ring_offset<hist_copies<KIND, IdxT, DF>()>() +
+                             tma_stages<hist_copies<KIND, IdxT, DF>()>() * kTmaChunk;
+      for (int s2 = 0; s2 < pre; ++s2) mbar_wait(fullb + 8u * s2, 0);
+    }
+    return;
+  }
   if (DF == 0 && redo && win_state == 1) return;           // pass 0 was done by the window pass
   const bool redo_buf = false;
   const int src1 = (FILTER || redo_buf) ? st->src1 : 0;    // Alg1 L7-8 (reading 6)
@@ -268,6 +282,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.err = &st->error;
   c.hist = sh_hist;
   c.ring = smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>();
+  c.pre_issued = (DF == 3 && TMA);
   c.wq = &sh_wq[HAS_Q ? warp : 0];
 
   if constexpr (FILTER && DH != 0) {
@@ -361,6 +376,26 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
     }
     st->ticket = 0;
   }
+  if constexpr (FILTER && DH != 0) {
+    // Finish in the scan: the candidates this pass stored (digit q-1 == j_{q-1}) are few, so the
+    // scanning CTA finishes the row from them right away (small_finish with digit q and the j_q just
+    // chosen) instead of leaving it to launch q+1 (which then returns at once, like every later one).
+    __syncthreads();  // the state update above
+    if (c.store && p.small_finish > 0 && p.trace == nullptr && st->stop1 == 0) {
+      const unsigned long long nb2 = __ldcg(c.bufc);
+      if (nb2 <= (unsigned long long)p.small_finish) {
+        PassCtx<U, IdxT> c2 = c;
+        c2.df = c.dh;
+        c2.tcode = st->tcode;
+        c2.tidx = st->tidx;
+        c2.bcin = c.bco;
+        c2.biin = c.bio;
+        c2.nbuf = nb2;
+        c2.srcL = false;
+        small_finish<KIND, IdxT, kBlock>(c2, st, (unsigned char*)sh_hist);
+      }
+    }
+  }
   dbg_stamp(p.trace, row, q, 3, 2, p.P);
 }
 
@@ -424,6 +459,7 @@ __device__ void select_digits(const W* a, int n, int& rank, W& prefix, W& mask, 
 // <= kBrute samples) or, for concentrated samples, 8-bit digits over the bin (select_digits).
 // Written for a short critical path: no loop carries a shared-memory load-atomic chain.
 constexpr int kBrute = 128;
+static_assert(kSampleBlock / 8 >= kBrute, "8 threads per bin member in the brute-force rank");
 
 template <typename W, int PER>
 __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo, int rhi, W pmin, int hb,
@@ -523,16 +559,24 @@ __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo,
     const int m = q ? m_hi : m_lo;
     int rk = q ? rk_hi : rk_lo;
     if (m <= kBrute) {
-      if ((int)threadIdx.x < m) {
-        const W x = reg[threadIdx.x];
-        int less = 0, eq = 0;
-        for (int j = 0; j < m; ++j) {
+      // rank of each of the m <= 128 bin members by counting: 8 threads per member, each over every
+      // 8th member, summed over the 8-lane group (m / 8 loads per thread instead of m)
+      const int e = (int)threadIdx.x >> 3, part = (int)threadIdx.x & 7;
+      const W x = (e < m) ? reg[e] : (W)0;
+      int less = 0, eq = 0;
+      if (e < m) {
+        for (int j = part; j < m; j += 8) {
           const W u = reg[j];
           less += u < x;
           eq += u == x;
         }
-        if (less <= rk && rk < less + eq) shw[4 + q] = x;
       }
+#pragma unroll
+      for (int o = 1; o < 8; o <<= 1) {
+        less += __shfl_xor_sync(kFull, less, o);
+        eq += __shfl_xor_sync(kFull, eq, o);
+      }
+      if (e < m && part == 0 && less <= rk && rk < less + eq) shw[4 + q] = x;
       __syncthreads();
       res[q] = shw[4 + q];
     } else {

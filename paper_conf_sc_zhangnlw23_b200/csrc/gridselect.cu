@@ -243,13 +243,16 @@ cudaError_t run_gridselect(const SelectArgs& a, void* ws, size_t ws_bytes, cudaS
   p.per_warp = (a.len + (int64_t)p.G * kGsWarps - 1) / ((int64_t)p.G * kGsWarps);
   cudaError_t e = cudaMemsetAsync(p.ticket, 0, (size_t)a.batch * 4, s);
   if (e != cudaSuccess) return e;
+  if (a.events && a.n_events > 0) cudaEventRecord((cudaEvent_t)a.events[0], s);
   switch (a.kind) {
-    case K_F32: return launch_gs<K_F32>(p, s);
-    case K_F16: return launch_gs<K_F16>(p, s);
-    case K_BF16: return launch_gs<K_BF16>(p, s);
-    case K_U32: return launch_gs<K_U32>(p, s);
+    case K_F32: e = launch_gs<K_F32>(p, s); break;
+    case K_F16: e = launch_gs<K_F16>(p, s); break;
+    case K_BF16: e = launch_gs<K_BF16>(p, s); break;
+    case K_U32: e = launch_gs<K_U32>(p, s); break;
+    default: return cudaErrorInvalidValue;
   }
-  return cudaErrorInvalidValue;
+  if (a.events && a.n_events > 1) cudaEventRecord((cudaEvent_t)a.events[1], s);
+  return e;
 }
 
 }  // namespace airtopk

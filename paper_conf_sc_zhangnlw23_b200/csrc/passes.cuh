@@ -189,8 +189,45 @@ struct PassCtx {
   unsigned long long* wmax;
   unsigned* hist;  // shared, kMaxBins * hist_copies() counters, zeroed by the caller
   unsigned ring;   // TMA streaming: shared-window address of the ring (after the histogram copies)
+  bool pre_issued; // TMA streaming: the ring's first stages were issued by tma_prologue (before pdl_wait)
   WarpQ<U, IdxT>* wq;
 };
+
+// First stages of the bulk-copy ring of a TMA pass over the input row (thread 0: barrier init + up to
+// NST copies). Depends only on the row pointer and the slice, so a kernel can issue it BEFORE
+// pdl_wait (the keys are never written by the select) and overlap the ring fill with the previous
+// launch. Returns the number of stages issued (thread 0).
+template <typename U, int HC, int BLOCK>
+__device__ __forceinline__ int tma_prologue(const U* rowp, int64_t len, int slice, int nslices, bool reverse,
+                                            unsigned ring) {
+  constexpr int VEC = 16 / sizeof(U);
+  constexpr int NST = tma_stages<HC>();
+  constexpr int NVT = (int)(kTmaChunk / 16 / BLOCK);
+  constexpr int64_t CV = (int64_t)BLOCK * NVT;
+  constexpr int NW = BLOCK / 32;
+  if (threadIdx.x != 0) return 0;
+  const uintptr_t mis = (uintptr_t)rowp & 15u;
+  const int64_t head = mis ? std::min<int64_t>(len, (int64_t)((16u - mis) / sizeof(U))) : 0;
+  const int64_t nvec = (len - head) / VEC;
+  const uint4* vp = (const uint4*)(rowp + head);
+  const unsigned fullb = ring + NST * kTmaChunk, emptyb = fullb + 8u * NST;
+  const int64_t nch = nvec / CV;
+  const int64_t mine = (nch > slice) ? (nch - 1 - slice) / nslices + 1 : 0;
+  const int64_t c0 = reverse ? (int64_t)slice + (mine - 1) * nslices : (int64_t)slice;
+  const int64_t sstep = (reverse ? -(int64_t)nslices : (int64_t)nslices) * CV;
+  const uint4* const src0 = vp + c0 * CV;
+  for (int st = 0; st < NST; ++st) {
+    mbar_init(fullb + 8u * st, 1);
+    mbar_init(emptyb + 8u * st, NW);
+  }
+  fence_mbar_init();
+  int st = 0;
+  for (; st < NST && st < mine; ++st) {
+    mbar_arrive_expect_tx(fullb + 8u * st, kTmaChunk);
+    bulk_g2s(ring + st * kTmaChunk, src0 + st * sstep, kTmaChunk, fullb + 8u * st);
+  }
+  return st;
+}
 
 // Runs the pass over this CTA's slice; the queues are flushed on return. Returns the number of
 // elements of the whole source (for the trace).
@@ -518,17 +555,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
       const int64_t cstep = c.reverse ? -(int64_t)c.nslices : (int64_t)c.nslices;
       const uint4* const src0 = vp + c0 * CV;
       const int64_t sstep = cstep * CV;  // in 16-byte vectors
-      if (tid == 0) {
-        for (int st = 0; st < NST; ++st) {
-          mbar_init(fullb + 8u * st, 1);
-          mbar_init(emptyb + 8u * st, NW);
-        }
-        fence_mbar_init();
-        for (int st = 0; st < NST && st < mine; ++st) {
-          mbar_arrive_expect_tx(fullb + 8u * st, kTmaChunk);
-          bulk_g2s(ring + st * kTmaChunk, src0 + st * sstep, kTmaChunk, fullb + 8u * st);
-        }
-      }
+      if (!c.pre_issued) tma_prologue<U, HC, BLOCK>(c.rowp, c.len, c.slice, c.nslices, c.reverse, ring);
       __syncthreads();
       int st = 0, pst = NST - 1;    // stage of this / the previous iteration
       unsigned ph = 0, pph = 1;     // their phase parities
