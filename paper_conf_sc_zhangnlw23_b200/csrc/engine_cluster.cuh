@@ -227,15 +227,14 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
         const int b0 = crank * seg;
         for (int b = tid; b < seg; b += kCBlock) {
           if (b0 + b < nb) {
-            unsigned x[kMaxCluster];
-#pragma unroll
-            for (int rr = 0; rr < kMaxCluster; ++rr) x[rr] = (rr < CS) ? cl.map_shared_rank(sh_hist, rr)[b0 + b] : 0u;
             unsigned v = 0;
+            for (int r0 = 0; r0 < CS; r0 += 4) {  // 4 DSMEM loads in flight (few registers)
+              unsigned x[4];
 #pragma unroll
-            for (int rr = 0; rr < kMaxCluster; ++rr) v += x[rr];
-#pragma unroll
-            for (int rr = 0; rr < kMaxCluster; ++rr)
-              if (rr < CS) cl.map_shared_rank(sh_seg, rr)[b0 + b] = v;
+              for (int i = 0; i < 4; ++i) x[i] = (r0 + i < CS) ? cl.map_shared_rank(sh_hist, r0 + i)[b0 + b] : 0u;
+              v += x[0] + x[1] + x[2] + x[3];
+            }
+            for (int rr = 0; rr < CS; ++rr) cl.map_shared_rank(sh_seg, rr)[b0 + b] = v;
           }
         }
         stamp(1);

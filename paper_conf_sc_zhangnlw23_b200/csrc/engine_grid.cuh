@@ -23,10 +23,11 @@
 // rule, so for radix-adversarial data the first index pass reads L once and buffers the ties.
 //
 // B200 mapping:
-//   * grid = batch x cpr CTAs of 512 threads, 3 CTAs/SM (444 CTAs fill the 148 SMs; measured
-//     faster than 4/SM), each CTA a contiguous slice of its row;
+//   * grid = batch x cpr CTAs of 512 threads, 2 CTAs/SM (296 CTAs fill the 148 SMs; measured
+//     faster than 3-4/SM), tile t of a row -> CTA t mod cpr (grid-stride: the CTAs of a row read one
+//     compact advancing region), or for a few long rows 1 CTA/SM streaming through a bulk-copy ring;
 //   * 4 x 128-bit ld.global.nc.L1::no_allocate loads in flight per thread (32 KiB per CTA tile);
-//   * odd passes walk their slice backwards so the tail the previous pass left in the 126 MB L2 is
+//   * odd passes walk their tiles backwards so the tail the previous pass left in the 126 MB L2 is
 //     consumed first;
 //   * 2048-bin shared histogram with plain shared atomics (measured at HBM speed on B200 even with
 //     32-way same-bin conflicts), merged with global red.add of the nonzero bins only;
@@ -161,7 +162,7 @@ constexpr int kMinBlocksFilter = AIRTOPK_SLOW_REG ? 2 : AIRTOPK_MINB;
 // Kernel q of the select. DF/DH: digit filtered / histogrammed (passes.cuh). DF == 3 is the
 // sample-guided window pass (q = 0); `redo` = the pass-0 histogram re-run over the window buffer.
 // TMA: the input row is streamed through per-warp shared rings by the bulk-copy engine (1 CTA/SM,
-// DESIGN.md "Kernels"); otherwise 4 x 16-byte register loads per thread (3 CTAs/SM).
+// DESIGN.md "Kernels"); otherwise 4 x 16-byte register loads per thread (2 CTAs/SM).
 // Debug timing of pass q (trace mode only; trace slot 7 + q of the row, zero-initialised):
 // [0] ~min CTA start, [1] max run_pass end, [2] max ticket arrival, [3] last CTA: scan done,
 // [4] CTA 0 start, [5] CTA 0 run_pass end
@@ -196,13 +197,6 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
   RowState* st = p.st + row;
-  // Window pass over bulk-copy rings: the ring's first stages depend only on the (read-only) keys, so
-  // they are issued before pdl_wait and fill while the sample kernel finishes.
-  int pre = 0;
-  if constexpr (DF == 3 && TMA)
-    pre = tma_prologue<typename KT<KIND>::U, hist_copies<KIND, IdxT, DF>(), kBlock>(
-        (const typename KT<KIND>::U*)p.keys + row * p.len, p.len, cta, p.cpr, false,
-        smem_addr(sh_hist) + (unsigned)tma_ring_offset<hist_copies<KIND, IdxT, DF>()>());
   pdl_wait();     // the previous pass's scan (row state, buffers) is complete and visible
   pdl_trigger();  // the next pass may be scheduled as our CTAs retire (hides launch latency)
 
@@ -211,14 +205,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   if (FILTER && stop1 != 0 && stop1 - 1 < q - 1) return;  // finished by an earlier early stop
   if (FILTER && q < st->npass) return;                     // digit done by the window pass (digit skip)
   const int win_state = (DF == 3 || (DF == 0 && redo)) ? st->win_state : 0;
-  if (DF == 3 && win_state != 1) {                         // no window: pass 0 will read L
-    if constexpr (DF == 3 && TMA) {  // (thread 0) the pre-issued copies must land before the CTA exits
-      const unsigned fullb = smem_addr(sh_hist) + (unsigned)tma_ring_offset<hist_copies<KIND, IdxT, DF>()>() +
-                             tma_stages<hist_copies<KIND, IdxT, DF>()>() * kTmaChunk;
-      for (int s2 = 0; s2 < pre; ++s2) mbar_wait(fullb + 8u * s2, 0);
-    }
-    return;
-  }
+  if (DF == 3 && win_state != 1) return;                   // no window: pass 0 will read L
   if (DF == 0 && redo && win_state == 1) return;           // pass 0 was done by the window pass
   const bool redo_buf = false;
   const int src1 = (FILTER || redo_buf) ? st->src1 : 0;    // Alg1 L7-8 (reading 6)
@@ -247,6 +234,10 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
     }
   }
   c.dh = digit_of(qs, KT<KIND>::R, p.IB);
+  // window pass: the members' histogram of the next digit too (used when all members turn out to
+  // share digit qs; only key digits: qs + 1 < code passes, else a copy of dh that is never used)
+  const bool two = (DF == 3) && (qs + 1 < code_passes(KT<KIND>::R));
+  c.dh2 = digit_of(two ? qs + 1 : qs, KT<KIND>::R, p.IB);
   c.df = digit_of(FILTER ? q - 1 : 0, KT<KIND>::R, p.IB);
   c.tcode = FILTER ? st->tcode : 0ull;
   c.tidx = FILTER ? st->tidx : 0ull;
@@ -282,7 +273,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.err = &st->error;
   c.hist = sh_hist;
   c.ring = smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>();
-  c.pre_issued = (DF == 3 && TMA);
+  c.pre_issued = false;
   c.wq = &sh_wq[HAS_Q ? warp : 0];
 
   if constexpr (FILTER && DH != 0) {
@@ -307,14 +298,24 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
 
   // ---- merge into the row histogram; the last CTA scans ----
   __syncthreads();
-  const Digit dh = c.dh;
+  Digit dh = c.dh;
   CountT* gh = (CountT*)p.ghist + ((size_t)row * 2 + (q & 1)) * kMaxBins;
-  const int nb = 1 << dh.width;
-  for (int i = tid; i < nb; i += kBlock) {
-    unsigned v = 0;
+  int nb = 1 << dh.width;
+  if constexpr (DF == 3) {  // two member histograms: digit qs -> slot 0, digit qs + 1 -> slot 1
+    CountT* gh1 = (CountT*)p.ghist + ((size_t)row * 2 + 1) * kMaxBins;
+    const int nb2 = 1 << c.dh2.width;
+    for (int i = tid; i < nb; i += kBlock)
+      if (sh_hist[i]) atomicAdd(&gh[i], (CountT)sh_hist[i]);
+    if (two)
+      for (int i = tid; i < nb2; i += kBlock)
+        if (sh_hist[kHistSlots + i]) atomicAdd(&gh1[i], (CountT)sh_hist[kHistSlots + i]);
+  } else {
+    for (int i = tid; i < nb; i += kBlock) {
+      unsigned v = 0;
 #pragma unroll
-    for (int h = 0; h < HC; ++h) v += sh_hist[i * HC + h];
-    if (v) atomicAdd(&gh[i], (CountT)v);
+      for (int h = 0; h < HC; ++h) v += sh_hist[i * HC + h];
+      if (v) atomicAdd(&gh[i], (CountT)v);
+    }
   }
   __syncthreads();  // the CTA's histogram merge / queue flushes precede thread 0's release
   dbg_stamp(p.trace, row, q, 2, 1, p.P);
@@ -335,7 +336,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
     Kin = kk - R;
     Cin = Wn;
     if (!window_ok) {  // miss: discard, the redo launch re-runs the paper's pass 1 over L
-      for (int i = tid; i < kMaxBins; i += kBlock) gh[i] = 0;
+      for (int i = tid; i < kMaxBins; i += kBlock) gh[i] = 0;  // (slot 1 is zeroed by the redo's scan)
       if (tid == 0) {
         st->win_state = 2;
         st->out_count = 0;
@@ -344,6 +345,17 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
         st->ticket = 0;
       }
       return;
+    }
+    // every member shares digit qs as well (their extremes agree on it): digit qs's histogram is a
+    // single bin, so continue from digit qs + 1's (slot 1) — launch qs + 1 then has nothing to do
+    if (two) {
+      const unsigned long long wmin = ~__ldcg(&st->win_nmin), wmax = __ldcg(&st->win_max);
+      if (Wn > 0 && (wmin >> dh.shift) == (wmax >> dh.shift)) {
+        qs += 1;
+        dh = c.dh2;
+        nb = 1 << dh.width;
+        gh = (CountT*)p.ghist + ((size_t)row * 2 + 1) * kMaxBins;
+      }
     }
   }
   const ScanResult r = scan_choose<kBlock>(
@@ -359,12 +371,16 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
       st->Cp = Cin;
       st->C = newC;
       st->K = newK;
-      if (DF == 3 && qs > 0) st->tcode = st->win_lo >> (dh.shift + dh.width) << (dh.shift + dh.width);
+      if (DF == 3 && qs > 0) {  // the digits above dh: common to every member (lo/hi, or their extremes)
+        const unsigned long long ref = (gh == (CountT*)p.ghist + ((size_t)row * 2 + 1) * kMaxBins)
+                                           ? ~__ldcg(&st->win_nmin) : st->win_lo;
+        st->tcode = ref >> (dh.shift + dh.width) << (dh.shift + dh.width);
+      }
       if (!dh.is_idx) st->tcode |= (unsigned long long)r.j << dh.shift;
       else st->tidx |= (unsigned long long)r.j << dh.shift;
       st->j = r.j;
       st->npass = qs + 1;
-      if (newK == newC) st->stop1 = q + 1;                             // early stop
+      if (newK == newC) st->stop1 = qs + 1;  // early stop; qs = the digit scanned (window skip)
       st->src1 = next_src1;
       st->buf_count[next_src1 == 1 ? 1 : 0] = 0;                        // next pass's output buffer
       if (r.total != Cin) st->error |= 4u;
@@ -375,26 +391,6 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
       }
     }
     st->ticket = 0;
-  }
-  if constexpr (FILTER && DH != 0) {
-    // Finish in the scan: the candidates this pass stored (digit q-1 == j_{q-1}) are few, so the
-    // scanning CTA finishes the row from them right away (small_finish with digit q and the j_q just
-    // chosen) instead of leaving it to launch q+1 (which then returns at once, like every later one).
-    __syncthreads();  // the state update above
-    if (c.store && p.small_finish > 0 && p.trace == nullptr && st->stop1 == 0) {
-      const unsigned long long nb2 = __ldcg(c.bufc);
-      if (nb2 <= (unsigned long long)p.small_finish) {
-        PassCtx<U, IdxT> c2 = c;
-        c2.df = c.dh;
-        c2.tcode = st->tcode;
-        c2.tidx = st->tidx;
-        c2.bcin = c.bco;
-        c2.biin = c.bio;
-        c2.nbuf = nb2;
-        c2.srcL = false;
-        small_finish<KIND, IdxT, kBlock>(c2, st, (unsigned char*)sh_hist);
-      }
-    }
   }
   dbg_stamp(p.trace, row, q, 3, 2, p.P);
 }
@@ -459,11 +455,12 @@ __device__ void select_digits(const W* a, int n, int& rank, W& prefix, W& mask, 
 // <= kBrute samples) or, for concentrated samples, 8-bit digits over the bin (select_digits).
 // Written for a short critical path: no loop carries a shared-memory load-atomic chain.
 constexpr int kBrute = 128;
+constexpr int kSampleHistCopies = 4;
 static_assert(kSampleBlock / 8 >= kBrute, "8 threads per bin member in the brute-force rank");
 
 template <typename W, int PER>
 __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo, int rhi, W pmin, int hb,
-                                 unsigned* hist /* 2048 */, unsigned* wsum /* 32 */, W* shw, int* cnt,
+                                 unsigned* hist /* 2048 x copies */, unsigned* wsum /* 32 */, W* shw, int* cnt,
                                  W& lo, W& hi) {
   constexpr int WB = 8 * (int)sizeof(W);
   if (hb <= 0) {  // all samples equal
@@ -475,15 +472,24 @@ __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo,
   const unsigned dmask = (1u << w) - 1u;
   const W mask = (hb >= WB) ? (W)0 : (W)(~(W)0 << hb);
   const W prefix = pmin & mask;
-  for (int i = threadIdx.x; i < 2048; i += blockDim.x) hist[i] = 0;
+  // kSampleHistCopies interleaved copies of each bin (lane % copies): uniform samples crowd a few
+  // bins (e.g. half of (0, 1] lies in one octave), and the copies cut the same-address serialisation
+  for (int i = threadIdx.x; i < 2048 * kSampleHistCopies; i += blockDim.x) hist[i] = 0;
   if (threadIdx.x < 2) cnt[threadIdx.x] = 0;
   __syncthreads();
+  const unsigned hcopy = (unsigned)(lane % kSampleHistCopies);
 #pragma unroll
   for (int t = 0; t < PER; ++t)
-    if (t < tv) atomicAdd(&hist[(unsigned)(v[t] >> sh) & dmask], 1u);
+    if (t < tv) atomicAdd(&hist[((unsigned)(v[t] >> sh) & dmask) * kSampleHistCopies + hcopy], 1u);
   __syncthreads();
+  auto binc = [&](unsigned b) {
+    unsigned x = 0;
+#pragma unroll
+    for (int h = 0; h < kSampleHistCopies; ++h) x += hist[b * kSampleHistCopies + h];
+    return x;
+  };
   // block scan: thread t owns bins 2t, 2t+1 (1024 threads)
-  const unsigned c0 = hist[2 * threadIdx.x], c1 = hist[2 * threadIdx.x + 1], tot = c0 + c1;
+  const unsigned c0 = binc(2 * threadIdx.x), c1 = binc(2 * threadIdx.x + 1), tot = c0 + c1;
   unsigned incl = tot;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
@@ -510,7 +516,7 @@ __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo,
   __syncthreads();
   const unsigned blo = (rlo >= 0) ? (unsigned)shw[0] : 0xffffffffu, bhi = (unsigned)shw[1];
   const int rk_lo = rlo - (int)shw[2], rk_hi = rhi - (int)shw[3];
-  const int m_lo = (rlo >= 0) ? (int)hist[blo] : 0, m_hi = (int)hist[bhi];
+  const int m_lo = (rlo >= 0) ? (int)binc(blo) : 0, m_hi = (int)binc(bhi);
   const W plo = prefix | ((W)blo << sh), phi = prefix | ((W)bhi << sh);
   if (sh == 0) {
     lo = plo;
@@ -592,13 +598,15 @@ __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo,
 constexpr int kSampleCTAs = 16;  // max CTAs per row issuing the scattered sample loads (one SM cannot
                                  // keep 16K independent DRAM loads in flight)
 
-template <int KIND>
+// ONE: one CTA per row (cps == 1; batches) — the samples stay in registers between the phases (a
+// separate instantiation: keeping them live in the multi-CTA variant costs it register spills)
+template <int KIND, bool ONE>
 __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p, int nsamp, int cps) {
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
   extern __shared__ __align__(16) unsigned char sample_smem[];
   W* scratch = (W*)sample_smem;  // nsamp entries: compacted bins of the rank selection (last CTA)
-  __shared__ unsigned hist[2048];
+  __shared__ unsigned hist[2048 * kSampleHistCopies];
   __shared__ unsigned wsum[32];
   __shared__ W shw[8];
   __shared__ int sh_cnt[4];
@@ -651,11 +659,11 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
       const int64_t pos = (int64_t)run * stride + (stride - kRun) / 2 + e;
       const bool ok = t < tmax && run < nruns && pos < p.len;
       const W code = ok ? (W)to_code_x<KIND>(x[t], xmask) : (W)0;
-      if (cps == 1) v[t] = code;  // one CTA per row: sample slot == run * kRun + e, kept in registers
+      if (ONE) v[t] = code;  // one CTA per row: sample slot == run * kRun + e, kept in registers
       else if (ok) samp[run * kRun + e] = code;
     }
   }
-  if (cps > 1) {
+  if (!ONE) {
     __syncthreads();
     if (threadIdx.x == 0) sh_last = (ticket_arrive(&st->ticket) == (unsigned)(cps - 1));
     __syncthreads();
@@ -665,7 +673,7 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
   // phase 2 (last CTA of the row): the window from the sample order statistics; the samples stay
   // in registers (16 per thread)
   const int tv = (nsamp - (int)threadIdx.x + kSampleBlock - 1) / kSampleBlock;  // valid v[t]: t < tv
-  if (cps > 1) {
+  if (!ONE) {
 #pragma unroll
     for (int t = 0; t < PER; ++t) v[t] = (t < tv) ? __ldcg(samp + t * kSampleBlock + threadIdx.x) : (W)0;
   }
@@ -805,13 +813,19 @@ cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, c
     using W = std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long, unsigned>;
     const size_t smem = (size_t)kMaxSamples * 4;  // 8-byte keys: nsamp <= kMaxSamples / 2
     static const cudaError_t attr =
-        cudaFuncSetAttribute(sample_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(sample_kernel<KIND, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    static const cudaError_t attr1 =
+        cudaFuncSetAttribute(sample_kernel<KIND, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (attr != cudaSuccess) return attr;
+    if (attr1 != cudaSuccess) return attr1;
     // CTAs per row: enough to spread a few rows' scattered loads over the SMs; one per row for
     // batches (each CTA then keeps up to 16 loads per thread in flight)
     const int cps = (int)std::max<int64_t>(1, std::min<int64_t>(kSampleCTAs, gp.nsms / batch));
-    cudaError_t es = launch_pdl(sample_kernel<KIND>, dim3((unsigned)(batch * cps)), dim3(kSampleBlock),
-                                (size_t)nsamp * sizeof(W), s, gp, nsamp, cps);
+    cudaError_t es = (cps == 1)
+        ? launch_pdl(sample_kernel<KIND, true>, dim3((unsigned)batch), dim3(kSampleBlock), (size_t)nsamp * sizeof(W),
+                     s, gp, nsamp, cps)
+        : launch_pdl(sample_kernel<KIND, false>, dim3((unsigned)(batch * cps)), dim3(kSampleBlock),
+                     (size_t)nsamp * sizeof(W), s, gp, nsamp, cps);
     if (es != cudaSuccess) return es;
     ev.record(ie++, s);
     cudaError_t e = launch_one<KIND, IdxT, 3, 0, HASIDX, TMA>(gp, grid, 0, 0, s);

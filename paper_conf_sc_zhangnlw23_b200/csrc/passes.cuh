@@ -51,7 +51,7 @@ constexpr unsigned kTmaChunk = AIRTOPK_TMA_CHUNK;    // bytes per bulk copy (one
 // dynamic + static shared memory per CTA is capped at 227 KiB; the static part (queues, scan
 // scratch) of the grid pass kernel stays below 20 KiB
 constexpr size_t kSmemCap = 232448;
-constexpr size_t kStaticSmemReserve = 20480;
+constexpr size_t kStaticSmemReserve = 19072;  // >= the largest static smem of a TMA pass kernel (ptxas: 18976)
 // Copies of the shared histogram in the filter passes: lane l counts into copy l % kHistCopies
 // (interleaved bin-major so copies of one bin sit in different banks); cuts the same-address
 // serialisation of shared atomics when many lanes hit a few bins (radix-adversarial passes).
@@ -64,8 +64,8 @@ template <int HC>
 constexpr size_t tma_ring_offset() { return ((size_t)kHistSlots * 4 * HC + 127) / 128 * 128; }
 template <int HC>
 constexpr int tma_stages() {
-  const size_t avail = kSmemCap - kStaticSmemReserve - tma_ring_offset<HC>() - 512;
-  const size_t s = avail / kTmaChunk;
+  const size_t avail = kSmemCap - kStaticSmemReserve - tma_ring_offset<HC>();
+  const size_t s = avail / (kTmaChunk + 16);  // stage + its two mbarriers
   return (int)(s < (size_t)kTmaStages ? s : (size_t)kTmaStages);
 }
 // dynamic shared memory of a TMA pass: [histogram copies][ring stages][full bars][empty bars]
@@ -90,7 +90,8 @@ struct WarpQ {
 template <int KIND, typename IdxT, int DF>
 __host__ __device__ constexpr int hist_copies() {
   using U = typename KT<KIND>::U;
-  return (DF == 0 || DF == 3) ? 1 : (sizeof(U) + sizeof(IdxT) <= 8 ? kHistCopies : 2);
+  // DF == 3 (window pass): two separate histograms of the window members, digits qs and qs + 1
+  return DF == 0 ? 1 : DF == 3 ? 2 : (sizeof(U) + sizeof(IdxT) <= 8 ? kHistCopies : 2);
 }
 
 // Store the n queued entries of a warp: results at out[br ...], candidates at buf[bc ...], in queue
@@ -164,6 +165,7 @@ struct PassCtx {
   int q;
   bool emit_all, do_hist, srcL, store, sel_min, reverse;
   Digit dh, df;
+  Digit dh2;        // DF == 3: the digit after dh (its member histogram at counter offset kHistSlots)
   unsigned long long tcode, tidx;  // fixed prefix bits after scan q-1
   // source: row L (slice `slice` of `nslices`) or the previous candidate buffer
   const U* rowp;
@@ -268,7 +270,10 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
   const W kx_nb = (W)1 << wq_;
   const W kx_flag = kx_S + ((emit_all || store) ? kx_nb : (W)0);  // fast-path flag threshold on y
   // shared-window address of this lane's histogram copy (c.hist is the dynamic smem base)
-  const unsigned hbase = (unsigned)__cvta_generic_to_shared(c.hist) + ((HC > 1) ? (unsigned)(lane % HC) * 4u : 0u);
+  const unsigned hbase =
+      (unsigned)__cvta_generic_to_shared(c.hist) + ((HC > 1 && DF != 3) ? (unsigned)(lane % HC) * 4u : 0u);
+  const int shh2 = c.dh2.shift;
+  const unsigned hmask2 = (1u << c.dh2.width) - 1u;
   const U xmask = sel_min ? (U)0 : (U)~(U)0;
   W wlo_seen = ~(W)0, whi_seen = 0;  // DF == 3: extremes of this thread's window members
 
@@ -352,6 +357,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
         wlo_seen = ((W)code < wlo_seen) ? (W)code : wlo_seen;
         whi_seen = ((W)code > whi_seen) ? (W)code : whi_seen;
         shared_inc(hbase + 4u * (unsigned)(((W)code >> shh) & hmask));
+        shared_inc(hbase + 4u * (unsigned)(kHistSlots + (((W)code >> shh2) & hmask2)));
       }
     }
     return w ? 0 : ((cd && store) ? 1 : 2);

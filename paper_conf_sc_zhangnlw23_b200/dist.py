@@ -6,9 +6,9 @@ Only the two natural partitionings exist (SURVEY.md §8(e
   rank; every rank selects its own rows. No data-path collective at all.
 * select_split_row — one huge row is split into contiguous shards; every rank selects the local
   top-K of its shard (row-local ties -> lowest local index == lowest global index inside the
-  shard), the K candidates of every rank are all-gathered (the ONE exchange step, NCCL
-  all_gather over NVLink), and a merge select over the world*K candidates, ties ranked by the
-  global index value, gives the global top-K on every rank. Exact: a global top-K element has
+  shard), the K candidates of every rank are all-gathered as packed (value bits, global index)
+  pairs (the ONE exchange step: one NCCL all_gather over NVLink), and a merge select over the
+  world*K candidates, ties ranked by the global index value, gives the global top-K on every rank. Exact: a global top-K element has
   fewer than K predecessors in (code, global index) order, hence fewer than K in its own shard,
   so it is in that shard's local top-K.
 
@@ -88,8 +88,12 @@ def select_split_row(x_shard, k: int, total_len: int, shard_offset: int, largest
         rank = dist.get_rank(group)
         gidx = torch.cat([gidx, total_len + rank * k + torch.arange(pad, dtype=torch.int64, device=gidx.device)])
     world = dist.get_world_size(group)
-    gv = _all_gather(_bits_view(v), group).view(v.dtype).reshape(-1)
-    gi = _all_gather(gidx, group).reshape(-1)
+    # ONE all-gather of packed (value bits, global index) pairs: [k, 2] int64 per rank
+    vb = _bits_view(v)
+    packed = torch.stack([vb.to(torch.int64), gidx], dim=1)
+    g = _all_gather(packed, group).reshape(-1, 2)
+    gv = g[:, 0].to(vb.dtype).view(v.dtype)
+    gi = g[:, 1].contiguous()
     idx_bits = max(1, int(total_len + world * k - 1).bit_length())
     mfn = merge_fn or (lambda a, b, kq, ib, lg: select_with_idx(a, b, kq, ib, largest=lg))
     return mfn(gv, gi, k, idx_bits, largest)

@@ -1,0 +1,9 @@
+#!/bin/bash
+mkdir -p gpurun_out
+rm -f gpurun_out/ab_*
+timeout 900 python -m pytest tests -m gpu -q -x --timeout 300 2>&1 | tail -15 > gpurun_out/pytest_gpu.log
+python __graft_entry__.py smoke > gpurun_out/smoke.log 2>&1
+CONFIGS="c3 c4 c2" bash tools/gpu_libab.sh "new::"
+python bench.py --config c1 --engine 4 --no-cpu --no-extras --e2e-steps 1 > gpurun_out/ab_c1_gs_1.json 2> gpurun_out/ab_c1_gs_1.err
+python tools/sample_timing.py c3 > gpurun_out/sample_timing.txt 2>&1
+python tools/pass_timing.py c4 > gpurun_out/pass_timing.txt 2>&1
