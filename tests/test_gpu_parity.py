@@ -422,3 +422,23 @@ def test_gridselect_sorted_output_and_c1():
     idx = i.reshape(-1)
     for a in range(31):
         assert vals[a] < vals[a + 1] or (vals[a] == vals[a + 1] and idx[a] < idx[a + 1])
+
+
+@pytest.mark.parametrize("dtn", ["f16", "bf16", "f64", "u32"])
+def test_other_dtypes_concentrated(dtn):
+    """Keys sharing long leading bit prefixes (c4-like adversarial M=20 values converted to each key
+    type) through the window path: window digit skips, member-extreme skips, mass ties."""
+    x = gen.adversarial_f32(77, 1 << 20, m_bits=20)
+    if dtn == "f64":
+        raw = x.astype(np.float64).view(np.uint64)
+    elif dtn == "f16":
+        raw = x.astype(np.float16).view(np.uint16)
+    elif dtn == "bf16":
+        raw = (x.view(np.uint32) >> 16).astype(np.uint16)  # truncation: the top 16 bits
+    else:
+        raw = x.view(np.uint32)
+    raw = raw.reshape(1, -1)
+    for k in (1, 1000, 50000):
+        for sm in (True, False):
+            v, i = gpu_select(raw, dtn, k, sm)
+            assert_parity(raw, dtn, k, sm, v, i)
