@@ -328,6 +328,8 @@ def main():
             ach = dom_alg / (per[dom] * 1e-3) / 1e9
             roofline = {"bound": "hbm", "kernel": names[dom], "achieved": ach, "peak": peak,
                         "peak_kind": peak_kind, "unit": "GB/s", "frac": ach / peak,
+                        "peak_note": "MEASURED_PEAKS hbm_gbs is a copy (read+write) rate; a read-only "
+                                     "stream can exceed it (frac slightly > 1)",
                         "traffic": load_traffic(cfg, dom, n_launch),
                         "alg_bytes_per_launch": dom_alg, "launch_ms": float(per[dom])}
         whole = (in_bytes + out_bytes) / (select_ms * 1e-3) / 1e9

@@ -46,8 +46,10 @@ def _check(status: int):
         raise AirTopKError(status, lib())
 
 
-def _opts(alpha=0, engine=ENGINE_AUTO, ctas_per_row=0, cluster_size=0, trace=None, events=None, window=0, tma=0):
+def _opts(alpha=0, engine=ENGINE_AUTO, ctas_per_row=0, cluster_size=0, trace=None, events=None, window=0, tma=0,
+          early_stop=0):
     o = Options()
+    o.early_stop = int(early_stop)
     o.window = int(window)
     o.tma = int(tma)
     o.alpha = int(alpha)
@@ -86,7 +88,7 @@ def describe(dtype, batch: int, length: int, k: int, alpha: int = 0, engine: int
 
 def select(x, k: int, largest: bool = False, *, alpha: int = 0, engine: int = ENGINE_AUTO,
            ctas_per_row: int = 0, cluster_size: int = 0, trace=None, events=None, window: int = 0,
-           tma: int = 0, workspace=None, out=None, stream=None):
+           tma: int = 0, early_stop: int = 0, workspace=None, out=None, stream=None):
     """Top-K of each row of `x` ([batch, len] or [len], contiguous CUDA tensor).
 
     Returns (values, indices): [batch, k] of x.dtype (raw bit copies) and int64 row-local indices,
@@ -107,7 +109,7 @@ def select(x, k: int, largest: bool = False, *, alpha: int = 0, engine: int = EN
         idx = torch.empty((batch, k), dtype=torch.int64, device=x2.device)
     else:
         vals, idx = out
-    o = _opts(alpha, engine, ctas_per_row, cluster_size, trace, events, window, tma)
+    o = _opts(alpha, engine, ctas_per_row, cluster_size, trace, events, window, tma, early_stop)
     need = int(lib().airtopk_workspace_bytes_ex(dt, batch, length, k, ctypes.byref(o)))
     if workspace is None and need:
         workspace = torch.empty(need, dtype=torch.uint8, device=x2.device)

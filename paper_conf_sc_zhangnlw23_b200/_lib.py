@@ -37,6 +37,7 @@ class Options(ctypes.Structure):
         ("events", ctypes.c_void_p),
         ("window", ctypes.c_int32),
         ("tma", ctypes.c_int32),
+        ("early_stop", ctypes.c_int32),
     ]
 
 

@@ -178,6 +178,7 @@ static airtopk_status validate(const SelectArgs& a) {
   if (a.engine < 0 || a.engine > 4 || a.engine == 3) return AIRTOPK_EINVAL;
   if (a.engine == 4 && !gridselect_supported(a)) return AIRTOPK_EINVAL;
   if (a.window < -1 || a.window > 1) return AIRTOPK_EINVAL;
+  if (a.early_stop < -1 || a.early_stop > 0) return AIRTOPK_EINVAL;
   if (a.in_idx && (a.batch != 1 || a.idx_bits < 1 || a.idx_bits > 63)) return AIRTOPK_EINVAL;
   return AIRTOPK_OK;
 }
@@ -228,6 +229,7 @@ static SelectArgs make_args(const void* keys, int dt, int64_t batch, int64_t len
     a.n_events = opt->events ? opt->n_events : 0;
     a.window = opt->window;
     a.tma = opt->tma;
+    a.early_stop = opt->early_stop;
   }
   if (a.alpha == 0) a.alpha = 128;
   return a;

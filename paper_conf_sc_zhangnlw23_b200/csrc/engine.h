@@ -22,6 +22,7 @@ struct SelectArgs {
   int cluster_size = 0;
   int window = 0;                   // sample-guided window: 0 auto, 1 on, -1 off
   int tma = 0;                      // bulk-copy streaming: 0 auto, 1 on, -1 off
+  int early_stop = 0;               // 0 on, -1 off (ablation)
   int64_t* trace = nullptr;
   void* const* events = nullptr;    // optional cudaEvent_t[n_events] recorded around launches
   int n_events = 0;

@@ -44,6 +44,7 @@ struct ClusterParams {
   void* bidx;    // per row: 2 x cap_alloc indices
   int64_t cap_rule, cap_alloc;
   int nclusters;
+  int early_stop;  // 0 on, -1 off (ablation)
   int tail;      // 1: continue rows after the grid engine's window pass
   int tail_q;    // tail mode: the grid engine ran passes q < tail_q after the window pass
   int timing_stride;  // int64 slots per CTA in `timing` (8; 24 with the merge-phase stamps, debug)
@@ -259,7 +260,7 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
       K = newK;
       if (!c.dh.is_idx) tcode |= (unsigned long long)j << c.dh.shift;
       else tidx |= (unsigned long long)j << c.dh.shift;
-      if (newK == newC) stop1 = q + 1;                                       // early stop
+      if (newK == newC && p.early_stop == 0) stop1 = q + 1;                                       // early stop
     }
     cl.sync();  // the cluster finishes the row before its buffers are reused
     ++n_rows;
@@ -303,6 +304,7 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   p.cap_rule = pl.cap_rule;
   p.cap_alloc = pl.cap_alloc;
   p.tail = tail;
+  p.early_stop = a.early_stop;
   p.tail_q = pl.tail_q;
   p.timing = a.trace;  // cluster engine: the trace buffer receives per-CTA timing instead
   p.timing_stride = getenv("AIRTOPK_CLUSTER_TIMING") ? 24 : 8;

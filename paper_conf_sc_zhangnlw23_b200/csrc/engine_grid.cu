@@ -63,6 +63,7 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t
   gp.trace = a.trace;
   gp.samp = base + pl.off_samp;
   gp.nsms = num_sms();
+  gp.early_stop = a.early_stop;
   {
     static const char* env = getenv("AIRTOPK_BUF_PER_CTA");  // A/B knob (0 = every CTA works)
     gp.buf_per_cta = env ? atoi(env) : kBufPerCTA;

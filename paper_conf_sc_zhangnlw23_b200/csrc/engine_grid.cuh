@@ -66,6 +66,7 @@ struct GridParams {
   void* samp;  // sample-guided window: [batch][nsamp] sampled codes
   int nsms;    // SMs of the device
   int small_finish;  // a buffer-source pass over <= this many entries finishes the row in one CTA
+  int early_stop;   // 0 on, -1 off (ablation)
   int buf_per_cta;  // buffer-source passes: CTAs beyond ceil(nbuf / buf_per_cta) exit at once (0: all work)
 };
 
@@ -380,7 +381,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
       else st->tidx |= (unsigned long long)r.j << dh.shift;
       st->j = r.j;
       st->npass = qs + 1;
-      if (newK == newC) st->stop1 = qs + 1;  // early stop; qs = the digit scanned (window skip)
+      if (newK == newC && p.early_stop == 0) st->stop1 = qs + 1;  // early stop; qs = the digit scanned (window skip)
       st->src1 = next_src1;
       st->buf_count[next_src1 == 1 ? 1 : 0] = 0;                        // next pass's output buffer
       if (r.total != Cin) st->error |= 4u;

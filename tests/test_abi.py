@@ -96,3 +96,12 @@ def test_gridselect_scope_validation_without_gpu():
     assert lib.airtopk_workspace_bytes_ex(3, 1, 1 << 16, 32, opts(4)) == 0       # f64 keys
     assert lib.airtopk_workspace_bytes_ex(0, 1, 1 << 16, 32, opts(3)) == 0       # no engine 3
     assert lib.airtopk_select_ex(p, 3, 1, 100, 10, 1, p, p, p, 1 << 30, None, opts(4)) == _lib.EINVAL
+
+
+def test_early_stop_option_validation_without_gpu():
+    lib = at.lib()
+    o = _lib.Options()
+    o.early_stop = -1
+    assert lib.airtopk_workspace_bytes_ex(0, 1, 1 << 16, 32, ctypes.byref(o)) > 0
+    o.early_stop = 2
+    assert lib.airtopk_workspace_bytes_ex(0, 1, 1 << 16, 32, ctypes.byref(o)) == 0

@@ -442,3 +442,17 @@ def test_other_dtypes_concentrated(dtn):
         for sm in (True, False):
             v, i = gpu_select(raw, dtn, k, sm)
             assert_parity(raw, dtn, k, sm, v, i)
+
+
+@pytest.mark.parametrize("engine", [0, 1, 2])
+@pytest.mark.parametrize("dist,batch,n,k", [("uniform", 1, 1 << 20, 1000), ("normal", 7, 1 << 16, 256),
+                                            ("adversarial", 1, 1 << 20, 5000)])
+def test_early_stop_off_invariance(engine, dist, batch, n, k):
+    """Early stopping only skips work: with it disabled (the Fig. 10 ablation) every
+    engine returns the same exact result, for the paper's passes and the window path."""
+    x = _keys(dist, 151, batch, n)
+    for window in (-1, 0):
+        if engine == 2 and window == 0:
+            continue
+        v, i = gpu_select(x, "f32", k, True, engine=engine, window=window, early_stop=-1)
+        assert_parity(x, "f32", k, True, v, i)

@@ -16,6 +16,7 @@ for c in c1 c2; do
 done
 python bench.py --config c3 --window -1 --no-cpu --no-extras --e2e-steps 1 > gpurun_out/bench_c3_paper.json 2> gpurun_out/bench_c3_paper.err
 timeout 600 python bench.py --config c5 --no-extras --e2e-steps 1 --cpu-budget 5 > gpurun_out/bench_c5.json 2> gpurun_out/bench_c5.err
+python tools/ablation.py > gpurun_out/ablation.txt 2>&1
 # launch lists (serialised, cold-cache): window path and paper path
 timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -c 40 --csv --log-file gpurun_out/launches_c3.csv python tools/prof_select.py --config c3 --reps 3 > /dev/null 2>&1
 timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -c 40 --csv --log-file gpurun_out/launches_c3_paper.csv python tools/prof_select.py --config c3 --reps 3 --window -1 > /dev/null 2>&1
