@@ -16,6 +16,7 @@
 // last-block scans dominate.
 #pragma once
 
+#include <algorithm>
 #include <cooperative_groups.h>
 #include <cstdlib>
 
@@ -30,7 +31,6 @@ namespace cg = cooperative_groups;
 constexpr int kCBlock = 512;
 constexpr int kCWarps = kCBlock / 32;
 constexpr int kMaxCluster = 16;
-
 struct ClusterParams {
   const void* keys;
   const int64_t* in_idx;
@@ -74,7 +74,7 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
   extern __shared__ unsigned sh_hist[];  // kHistSlots counters
   __shared__ WarpQ<U, IdxT> sh_wq[kCWarps];
   __shared__ ClusterShared cs;
-  __shared__ unsigned sh_seg[kMaxBins];  // the cluster's merged histogram (each CTA's copy)
+  __shared__ __align__(16) unsigned sh_seg[kMaxBins];  // the cluster's merged histogram (each CTA's copy)
 
   cg::cluster_group cl = cg::this_cluster();
   const int CS = (int)cl.num_blocks();

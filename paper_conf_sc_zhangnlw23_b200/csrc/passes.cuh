@@ -753,4 +753,80 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
   return nread;
 }
 
+// Single-CTA finish of a row: pass q reads a buffer of n <= kSmallFinish
+// entries, all sharing the prefix of digits < q-1. Its filter of digit q-1 (Alg1 L15-22) emits the
+// entries below the target digit j; among the C entries with digit q-1 == j the K smallest composite
+// keys (code, index) — the lowest-index rule of reading 1 — are the rest of the result. With C small
+// these are found by rank counting in shared memory instead of the remaining radix passes
+// (rank(e) = #{e' : (code', idx') < (code, idx)}; keys are unique, so exactly K ranks are < K).
+// The caller ends the row (grid engine: stop1 = q, so every later launch returns at once).
+// sc, si: shared arrays of at least c.nbuf codes / indices.
+template <int KIND, typename IdxT, int BLOCK>
+__device__ void small_finish(const PassCtx<typename KT<KIND>::U, IdxT>& c, unsigned long long Kr,
+                             typename KT<KIND>::U* sc, IdxT* si) {
+  using U = typename KT<KIND>::U;
+  using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
+  __shared__ unsigned s_m;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int n = (int)c.nbuf;
+  const Digit df = c.df;
+  const unsigned long long jprev = (df.is_idx ? c.tidx : c.tcode) >> df.shift & ((1ull << df.width) - 1ull);
+  if (tid == 0) s_m = 0;
+  __syncthreads();
+  auto emit = [&](bool pred, U code, IdxT idx) {  // warp-aggregated result append
+    const unsigned m = __ballot_sync(kFull, pred);
+    if (!m) return;
+    unsigned long long b = 0;
+    if (lane == 0) b = atomicAdd(c.outc, (unsigned long long)__popc(m));
+    b = __shfl_sync(kFull, b, 0);
+    if (pred) {
+      const unsigned long long pos = b + __popc(m & lanemask_lt());
+      if (pos < c.kk) {
+        c.ov[pos] = from_code<KIND>(code, c.sel_min);
+        c.oi[pos] = (int64_t)idx;
+      } else {
+        atomicOr(c.err, 1u);
+      }
+    }
+  };
+  for (int b0 = 0; b0 < n; b0 += BLOCK) {
+    const int i = b0 + tid;
+    const bool valid = i < n;
+    const U code = valid ? c.bcin[i] : (U)0;
+    const IdxT idx = valid ? c.biin[i] : (IdxT)0;
+    const unsigned long long d = (df.is_idx ? (unsigned long long)idx : (unsigned long long)(W)code) >> df.shift &
+                                 ((1ull << df.width) - 1ull);
+    emit(valid && d < jprev, code, idx);
+    const bool eq = valid && d == jprev;
+    const unsigned m = __ballot_sync(kFull, eq);
+    unsigned b = 0;
+    if (lane == 0 && m) b = atomicAdd(&s_m, (unsigned)__popc(m));
+    b = __shfl_sync(kFull, b, 0);
+    if (eq) {
+      const unsigned pos = b + __popc(m & lanemask_lt());
+      sc[pos] = code;
+      si[pos] = idx;
+    }
+  }
+  __syncthreads();
+  const int m = (int)s_m;
+  for (int b0 = 0; b0 < m; b0 += BLOCK) {
+    const int i = b0 + tid;
+    bool sel = false;
+    U code = 0;
+    IdxT idx = 0;
+    if (i < m) {
+      code = sc[i];
+      idx = si[i];
+      unsigned long long rank = 0;
+      if ((unsigned long long)m > Kr)
+        for (int t = 0; t < m; ++t) rank += (sc[t] < code) || (sc[t] == code && si[t] < idx);
+      sel = rank < Kr;
+    }
+    emit(sel, code, idx);
+  }
+  if (tid == 0 && (unsigned long long)m < Kr) atomicOr(c.err, 4u);
+  __syncthreads();
+}
+
 }  // namespace airtopk
