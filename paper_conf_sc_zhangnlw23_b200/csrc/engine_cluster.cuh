@@ -181,7 +181,6 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
       c.err = &st->error;
       c.hist = sh_hist;
       c.ring = 0;
-      c.pre_issued = false;
       c.wq = &sh_wq[warp];
       const bool hist_on = c.do_hist || DF == 0;
       if (hist_on) {

@@ -65,8 +65,6 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t
   gp.nsms = num_sms();
   gp.early_stop = a.early_stop;
   {
-    static const char* env = getenv("AIRTOPK_BUF_PER_CTA");  // A/B knob (0 = every CTA works)
-    gp.buf_per_cta = env ? atoi(env) : kBufPerCTA;
     static const char* env2 = getenv("AIRTOPK_SMALL_FINISH");  // A/B knob (0 = off)
     gp.small_finish = env2 ? std::min(atoi(env2), kSmallFinish) : kSmallFinish;
   }

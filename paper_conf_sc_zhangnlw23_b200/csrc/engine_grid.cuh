@@ -67,7 +67,6 @@ struct GridParams {
   int nsms;    // SMs of the device
   int small_finish;  // a buffer-source pass over <= this many entries finishes the row in one CTA
   int early_stop;   // 0 on, -1 off (ablation)
-  int buf_per_cta;  // buffer-source passes: CTAs beyond ceil(nbuf / buf_per_cta) exit at once (0: all work)
 };
 
 constexpr int kBlock = 512;
@@ -75,7 +74,6 @@ constexpr int kBlock = 512;
 #define AIRTOPK_GRID_BU 4
 #endif
 constexpr int kGridBU = AIRTOPK_GRID_BU;  // buffer entries per thread per iteration of a buffer pass
-constexpr int kBufPerCTA = 0;  // buffer entries per working CTA of a buffer-source pass (0: all; measured: fewer CTAs are slower)
 constexpr int kSmallFinish = 1024;  // max buffer entries of the single-CTA finish (shared memory)
 
 constexpr int kWarps = kBlock / 32;
@@ -134,14 +132,13 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   const int win_state = (DF == 3 || (DF == 0 && redo)) ? st->win_state : 0;
   if (DF == 3 && win_state != 1) return;                   // no window: pass 0 will read L
   if (DF == 0 && redo && win_state == 1) return;           // pass 0 was done by the window pass
-  const bool redo_buf = false;
-  const int src1 = (FILTER || redo_buf) ? st->src1 : 0;    // Alg1 L7-8 (reading 6)
+  const int src1 = FILTER ? st->src1 : 0;    // Alg1 L7-8 (reading 6)
   const int sslot = (src1 == 1) ? 1 : 0;                   // candidate buffer this pass writes
   PassCtx<U, IdxT> c;
   c.q = q;
   c.emit_all = FILTER && ((stop1 != 0 && stop1 - 1 == q - 1) || DH == 0);
   c.do_hist = (DH != 0) && !c.emit_all;
-  const unsigned long long Cprev = (FILTER || redo_buf) ? st->C : (unsigned long long)p.len;  // C_{q-1}
+  const unsigned long long Cprev = FILTER ? st->C : (unsigned long long)p.len;  // C_{q-1}
   c.srcL = (src1 == 0);
   if (DF == 3) c.store = (win_state == 1);
   else c.store = c.do_hist && FILTER && (Cprev <= (unsigned long long)p.cap_rule);  // Alg1 L17
@@ -175,16 +172,8 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.rowp = (const U*)p.keys + row * p.len;
   c.rowi = HASIDX ? p.in_idx + row * p.len : nullptr;
   c.len = p.len;
-  // A pass over a (small) candidate buffer needs few CTAs: only the first `act` take part (fewer
-  // same-address histogram merges and ticket arrivals); the others leave right away.
-  int act = p.cpr;
-  if (src1 > 0 && p.buf_per_cta > 0) {
-    const unsigned long long nb = st->buf_count[src1 - 1];
-    act = (int)min((unsigned long long)p.cpr, max(1ull, (nb + p.buf_per_cta - 1) / (unsigned long long)p.buf_per_cta));
-    if (cta >= act) return;
-  }
   c.slice = cta;
-  c.nslices = act;
+  c.nslices = p.cpr;
   const int islot = src1 > 0 ? src1 - 1 : 0;
   c.bcin = (const U*)p.bcode + ((size_t)islot * p.batch + row) * p.cap_alloc;
   c.biin = (const IdxT*)p.bidx + ((size_t)islot * p.batch + row) * p.cap_alloc;
@@ -200,7 +189,6 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.err = &st->error;
   c.hist = sh_hist;
   c.ring = smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>();
-  c.pre_issued = false;
   c.wq = &sh_wq[HAS_Q ? warp : 0];
 
   if constexpr (FILTER && DH != 0) {
@@ -250,12 +238,12 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   }
   __syncthreads();  // the CTA's histogram merge / queue flushes precede thread 0's release
   dbg_stamp(p.trace, row, q, 2, 1, p.P);
-  if (tid == 0) sh_last = (ticket_arrive(&st->ticket) == (unsigned)(act - 1));
+  if (tid == 0) sh_last = (ticket_arrive(&st->ticket) == (unsigned)(p.cpr - 1));
   __syncthreads();
   if (!sh_last) return;
 
   const unsigned long long kk = (unsigned long long)p.k;
-  unsigned long long Kin = (FILTER || redo_buf) ? st->K : kk;
+  unsigned long long Kin = FILTER ? st->K : kk;
   unsigned long long Cin = Cprev;  // elements counted by this histogram
   bool window_ok = false;
   if constexpr (DF == 3) {

@@ -191,14 +191,11 @@ struct PassCtx {
   unsigned long long* wmax;
   unsigned* hist;  // shared, kMaxBins * hist_copies() counters, zeroed by the caller
   unsigned ring;   // TMA streaming: shared-window address of the ring (after the histogram copies)
-  bool pre_issued; // TMA streaming: the ring's first stages were issued by tma_prologue (before pdl_wait)
   WarpQ<U, IdxT>* wq;
 };
 
 // First stages of the bulk-copy ring of a TMA pass over the input row (thread 0: barrier init + up to
-// NST copies). Depends only on the row pointer and the slice, so a kernel can issue it BEFORE
-// pdl_wait (the keys are never written by the select) and overlap the ring fill with the previous
-// launch. Returns the number of stages issued (thread 0).
+// NST copies). Returns the number of stages issued (thread 0).
 template <typename U, int HC, int BLOCK>
 __device__ __forceinline__ int tma_prologue(const U* rowp, int64_t len, int slice, int nslices, bool reverse,
                                             unsigned ring) {
@@ -561,7 +558,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
       const int64_t cstep = c.reverse ? -(int64_t)c.nslices : (int64_t)c.nslices;
       const uint4* const src0 = vp + c0 * CV;
       const int64_t sstep = cstep * CV;  // in 16-byte vectors
-      if (!c.pre_issued) tma_prologue<U, HC, BLOCK>(c.rowp, c.len, c.slice, c.nslices, c.reverse, ring);
+      tma_prologue<U, HC, BLOCK>(c.rowp, c.len, c.slice, c.nslices, c.reverse, ring);
       __syncthreads();
       int st = 0, pst = NST - 1;    // stage of this / the previous iteration
       unsigned ph = 0, pph = 1;     // their phase parities

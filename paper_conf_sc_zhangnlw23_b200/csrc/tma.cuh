@@ -53,29 +53,8 @@ __device__ __forceinline__ bool mbar_try_wait(unsigned bar, unsigned parity) {
   return ok != 0;
 }
 
-#ifndef AIRTOPK_MBAR_HINT
-#define AIRTOPK_MBAR_HINT 0  // suspend-time hint (ns) of the consumers' waits; 0: plain polling
-#endif
-
-// try_wait with a suspend-time hint: the waiting thread sleeps until the phase completes (or the hint
-// elapses) instead of re-issuing the poll, leaving issue slots to the warps that have data
-__device__ __forceinline__ bool mbar_try_wait_hint(unsigned bar, unsigned parity, unsigned ns) {
-  unsigned ok;
-  asm volatile(
-      "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n selp.u32 %0, 1, 0, p;\n}"
-      : "=r"(ok)
-      : "r"(bar), "r"(parity), "r"(ns)
-      : "memory");
-  return ok != 0;
-}
-
 __device__ __forceinline__ void mbar_wait(unsigned bar, unsigned parity) {
-  if (AIRTOPK_MBAR_HINT > 0) {
-    while (!mbar_try_wait_hint(bar, parity, (unsigned)AIRTOPK_MBAR_HINT)) {
-    }
-  } else {
-    while (!mbar_try_wait(bar, parity)) {
-    }
+  while (!mbar_try_wait(bar, parity)) {
   }
 }
 
