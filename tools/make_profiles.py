@@ -32,7 +32,8 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
 
 def main(rnd):
     os.makedirs(PROF, exist_ok=True)
-    traffic = {}
+    tpath = os.path.join(PROF, "traffic_launches.json")
+    traffic = json.load(open(tpath)) if os.path.exists(tpath) else {}  # merged: configs not re-measured stay
     for f in sorted(glob.glob(os.path.join(OUT, "launches_*.csv"))):
         cfg = os.path.basename(f)[len("launches_"):-4]
         try:
@@ -67,6 +68,8 @@ def main(rnd):
                     lines.append(f"   {k:62s} {r[h.index(k)]} {rows[1][h.index(k)]}")
         open(os.path.join(PROF, f"{rnd}_ncu_{name}.txt"), "w").write("\n".join(lines) + "\n")
     for f in sorted(glob.glob(os.path.join(OUT, "bench_*.json"))):
+        if "sanity" in f:
+            continue
         txt = open(f).read().strip()
         if txt:
             open(os.path.join(PROF, f"{rnd}_{os.path.basename(f)}"), "w").write(txt.splitlines()[-1] + "\n")
