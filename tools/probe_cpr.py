@@ -1,4 +1,5 @@
-"""Select time vs CTAs per row (grid engine), for batched configs:  python tools/probe_cpr.py c2 2 4 8 16 32"""
+"""Select time vs CTAs per row (grid engine), for batched configs:  python tools/probe_cpr.py c2 2 4 8 16 32
+(PROBE_TMA=1 forces the bulk-copy streaming path)"""
 import os
 import sys
 
@@ -19,9 +20,9 @@ for cpr in [int(a) for a in sys.argv[2:]]:
             flush.fill_(1)
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
-            at.select(x, c["k"], ctas_per_row=cpr)
+            at.select(x, c["k"], ctas_per_row=cpr, tma=int(os.environ.get("PROBE_TMA", "0")))
             e1.record()
             e1.synchronize()
             if it >= 5:
                 tot += e0.elapsed_time(e1)
-        print(f"{cfg} cpr={cpr:4d} rep={rep} {tot / 35 * 1e3:8.1f} us", flush=True)
+        print(f"{cfg} tma={os.environ.get('PROBE_TMA', '0')} cpr={cpr:4d} rep={rep} {tot / 35 * 1e3:8.1f} us", flush=True)
