@@ -44,7 +44,7 @@ CFG = {
     # one 2^33 row: on one GPU the whole row (64-bit index path), at N ranks a 2^33/N shard each
     "c5": dict(batch=1, n=1 << 33, k=1 << 16, dist="uniform"),
 }
-DEFAULT_STEPS = {"c1": 200, "c2": 100, "c3": 60, "c4": 60, "c5": 10}
+DEFAULT_STEPS = {"c1": 500, "c2": 300, "c3": 200, "c4": 200, "c5": 10}  # timed regions >= ~0.1 s (clock samples)
 
 
 def log(*a):
