@@ -107,7 +107,8 @@ typedef struct {
   int32_t window;       /* sample-guided window pass: 0 = auto (grid engine,
                            len >= 2^18), 1 = on, -1 = off (the paper's passes only). Exact either way. */
   int32_t tma;          /* grid engine streaming: 0 = auto (bulk-copy rings for a few long rows), 1 = bulk
-                           copies (cp.async.bulk + mbarrier per-warp rings), -1 = register loads. */
+                           copies (cp.async.bulk into a per-CTA ring of 32 KiB stages, mbarrier handshake),
+                           -1 = register loads. */
   int32_t early_stop;   /* early stopping: 0 = on (default), -1 = off (the Fig. 10 ablation:
                            the passes continue after K == C; results identical). */
 } airtopk_options;
