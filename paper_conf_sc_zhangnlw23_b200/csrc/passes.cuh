@@ -283,7 +283,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
   W wx = 0;
   if constexpr (DF == 3) {
     constexpr W S = (W)((W)1 << (KT<KIND>::R - 1));
-    constexpr W ones = (W)(~(U)0);
+    constexpr W ones = (W)(U)~(U)0;  // (U) again: ~ promotes 16-bit keys to int
     if constexpr (KT<KIND>::IEEE) {
       if (sel_min) wx = (whi >= S) ? S : ones;
       else wx = (whi < S) ? (W)(ones ^ S) : (W)0;

@@ -456,3 +456,25 @@ def test_early_stop_off_invariance(engine, dist, batch, n, k):
             continue
         v, i = gpu_select(x, "f32", k, True, engine=engine, window=window, early_stop=-1)
         assert_parity(x, "f32", k, True, v, i)
+
+
+@pytest.mark.parametrize("dtn", ["f16", "bf16"])
+@pytest.mark.parametrize("front", [False, True])
+@pytest.mark.parametrize("select_min", [True, False])
+def test_window_16bit_extreme_codes(dtn, front, select_min):
+    """Regression (found by tests/fuzz_gpu.py): 16-bit keys whose selected code is the extreme one
+    (-NaN with full payload for select-min: code 0), ties partly in the scalar tail of a row whose
+    length is not a multiple of 8, through the window pass. The raw-bit window test must widen the
+    16-bit all-ones mask without integer promotion."""
+    n = 1510669
+    raw = np.sort(gen.u64(5, n).astype(np.uint16))
+    if not select_min:
+        raw = raw[::-1].copy()
+    if front:
+        cnt = int((raw == raw[-1]).sum())
+        raw = np.concatenate([raw[-cnt:], raw[:-cnt]])
+    raw = raw.reshape(1, n)
+    for k in (1, 2, 17):
+        for window in (0, 1):
+            v, i = gpu_select(raw, dtn, k, select_min, window=window)
+            assert_parity(raw, dtn, k, select_min, v, i)
