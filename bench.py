@@ -124,9 +124,42 @@ def n_passes(n: int, R: int = 32):
 
 
 # ----------------------------------------------------------------------------- reference arm / CPU baseline
+METRIC = "top-K elements/s and achieved HBM GB/s vs B200 peak (N=2^30,K=2^20; b=100)"
+
+
+def cpu_info():
+    """lscpu model name, usable cores and OMP_NUM_THREADS of this host."""
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ln.lower().startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    try:
+        usable = len(os.sched_getaffinity(0))
+    except Exception:
+        usable = os.cpu_count()
+    return {"lscpu_model": model, "nproc": usable, "cpu_count": os.cpu_count(),
+            "OMP_NUM_THREADS": os.environ.get("OMP_NUM_THREADS")}
+
+
+def _time_oracle(fn, budget_s, min_reps=1):
+    reps, t0 = 0, time.perf_counter()
+    while True:
+        r = fn()
+        reps += 1
+        el = time.perf_counter() - t0
+        if reps >= min_reps and el >= budget_s:
+            return reps, el, r
+
+
 def cpu_sample_run(cfg_name: str, budget_s: float):
-    """Time the CPU oracle (oracle.topk_nth, single thread, as it stands) on a bounded sample of the
-    workload: same distribution and K/N ratio, N_s = min(N, 2^26) per row."""
+    """Time the CPU oracle as it stands on a bounded sample of the workload (same distribution and
+    K/N ratio, N_s = min(N, 2^26) per row): the all-cores variant (oracle.topk_nth_mt, OpenMP) is
+    the reported value; the single-core oracle.topk_nth is timed beside it."""
     import oracle
     c = CFG[cfg_name]
     ns = min(c["n"], 1 << 26)
@@ -135,34 +168,69 @@ def cpu_sample_run(cfg_name: str, budget_s: float):
     x = host_keys(cfg_name, ns, rows)
     oracle.build()
     oracle.topk_nth(x[:1, : min(ns, 1 << 16)], min(ks, 1 << 16))  # load / warm
-    t0 = time.perf_counter()
-    reps = 0
-    while True:
-        oracle.topk_nth(x, ks)
-        reps += 1
-        el = time.perf_counter() - t0
-        if el >= budget_s:
-            break
-    value = reps * rows * ns / el
-    return {"value": value, "unit": "elements/s", "cores": 1, "kind": "oracle",
-            "sample": f"{reps} x oracle.topk_nth on {rows} x 2^{int(math.log2(ns))} {c['dist']} f32, K={ks} "
-                      f"(same K/N as {cfg_name}), {el:.1f} s single-threaded std::nth_element"}
+    reps, el, r = _time_oracle(lambda: oracle.topk_nth_mt(x, ks), budget_s / 2)
+    threads = r[2]
+    reps1, el1, _ = _time_oracle(lambda: oracle.topk_nth(x, ks), budget_s / 2)
+    info = cpu_info()
+    return {"value": reps * rows * ns / el, "unit": "elements/s", "cores": threads, "kind": "oracle",
+            "variant": "oracle.topk_nth_mt (OpenMP chunks + candidate merge, all cores)",
+            "single_core": {"value": reps1 * rows * ns / el1, "cores": 1, "variant": "oracle.topk_nth",
+                            "reps": reps1, "seconds": el1},
+            "sample": f"{reps} x oracle.topk_nth_mt on {rows} x 2^{int(math.log2(ns))} {c['dist']} f32, K={ks} "
+                      f"(same K/N as {cfg_name}), {el:.1f} s on {threads} threads",
+            **info}
 
 
 def run_reference(args, rank):
+    """The reference arm: this tier's reference is the CPU oracle (the paper ships no code). It runs
+    the repo arm's exact metric and workload (the real config input, e.g. c3 = 2^30 keys) on the
+    host cores: one untimed warm-up select, then as many timed selects as fit in --ref-budget
+    seconds (at least one); `steps` = the selects actually timed."""
     if rank != 0:
         return
+    import oracle
     cfg = args.config
     c = CFG[cfg]
-    cb = cpu_sample_run(cfg, args.ref_budget)
-    line = {"impl": "reference", "metric": f"top-K elements/s ({cfg})", "value": cb["value"], "unit": "elements/s",
-            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": c["batch"] * c["n"] / cb["value"] * 1e3, "higher_is_better": True,
+    oracle.build()
+    t0 = time.perf_counter()
+    x = host_keys(cfg, c["n"], c["batch"])
+    gen_s = time.perf_counter() - t0
+    oracle.topk_nth_mt(x, c["k"])  # warm-up (allocation, page faults)
+    reps, el, r = _time_oracle(lambda: oracle.topk_nth_mt(x, c["k"]), args.ref_budget)
+    threads = r[2]
+    value = reps * c["batch"] * c["n"] / el
+    cb = {"value": value, "unit": "elements/s", "cores": threads, "kind": "oracle",
+          "variant": "oracle.topk_nth_mt (OpenMP chunks + candidate merge, all cores)",
+          "sample": f"the full {cfg} input ({c['batch']} x {c['n']} {c['dist']} f32, K={c['k']}): "
+                    f"{reps} timed selects in {el:.1f} s after 1 warm-up (input generated in {gen_s:.1f} s)",
+          **cpu_info()}
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "elements/s",
+            "n_gpus": args.gpus, "steps": reps, "warmup": 1, "steps_requested": args.steps,
+            "ms_per_step": el / reps * 1e3, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": cfg, "batch": c["batch"], "n": c["n"], "k": c["k"], "dist": c["dist"]},
-            "cpu_baseline": cb, "e2e": {"value": cb["value"], "unit": "elements/s", "h2d_bytes_per_step": 0,
+            "cpu_baseline": cb, "e2e": {"value": value, "unit": "elements/s", "h2d_bytes_per_step": 0,
                                         "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def maybe_relaunch(args):
+    """`bench.py --gpus N` (N > 1) outside torchrun: re-exec under torch.distributed.run with N
+    ranks on this node (the driver's own launch sets WORLD_SIZE, so it runs directly)."""
+    if args.gpus <= 1 or "WORLD_SIZE" in os.environ or args.impl == "reference":
+        return
+    import socket
+    so = socket.socket()
+    so.bind(("127.0.0.1", 0))
+    port = so.getsockname()[1]
+    so.close()
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")          # communicator lines show nranks / NVLS
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    log("relaunching under torchrun:", " ".join(cmd))
+    os.execve(sys.executable, cmd, env)
 
 
 # ----------------------------------------------------------------------------- our arm
@@ -176,7 +244,7 @@ def main():
     ap.add_argument("--no-extras", action="store_true", help="skip the c1/c2/c4 side measurements")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--cpu-budget", type=float, default=10.0)
-    ap.add_argument("--ref-budget", type=float, default=20.0)
+    ap.add_argument("--ref-budget", type=float, default=30.0)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--engine", type=int, default=0, help="0 auto, 1 grid, 2 cluster (ablations)")
     ap.add_argument("--dtype", default="f32", choices=["f32", "f16", "bf16", "f64", "u32"],
@@ -189,6 +257,7 @@ def main():
     if args.steps is None:
         args.steps = DEFAULT_STEPS[args.config]
     args.warmup = max(3, args.warmup)
+    maybe_relaunch(args)
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -253,13 +322,25 @@ def main():
     stream = torch.cuda.current_stream(dev)
     ev_sets = []
 
+    total_len = (c["n"] if cfg == "c5" else world * n)
+    if split:  # gather buffers reused every step; the shard select writes into slot `rank` in place
+        gbuf = (torch.empty(world * k, dtype=kdt, device=dev), torch.empty(world * k, dtype=torch.int64, device=dev))
+        ws_shard = torch.empty(max(1, at.lib().airtopk_workspace_bytes_shard(at.dtype_code(kdt), n, k)),
+                               dtype=torch.uint8, device=dev)
+        mbits = at.merge_idx_bits(total_len, world, k)
+        ws_merge = torch.empty(max(1, at.lib().airtopk_workspace_bytes_with_idx(at.dtype_code(kdt), world * k, k,
+                                                                                  mbits)), dtype=torch.uint8, device=dev)
+        mout = (torch.empty(k, dtype=kdt, device=dev), torch.empty(k, dtype=torch.int64, device=dev))
+
     def step(events=None):
-        v, i = at.select(xd, k, workspace=ws, out=(ov, oi), events=events, **sel_opts)
         if split:
-            gv, gi = atdist.select_split_row(xd.reshape(-1), k, total_len=world * n, shard_offset=rank * n,
-                                             select_fn=lambda t, kk, lg: (v.reshape(-1), i.reshape(-1)))
-            return gv, gi
-        return v, i
+            return atdist.select_split_row(
+                xd.reshape(-1), k, total_len=total_len, shard_offset=rank * n, buffers=gbuf,
+                shard_fn=lambda t, kk, off, pb, lg, out: at.select_shard(t, kk, off, pb, largest=lg, out=out,
+                                                                         workspace=ws_shard),
+                merge_fn=lambda a, b, kq, ib, lg: at.select_with_idx(a, b, kq, ib, largest=lg, workspace=ws_merge,
+                                                                     out=mout))
+        return at.select(xd, k, workspace=ws, out=(ov, oi), events=events, **sel_opts)
 
     for _ in range(args.warmup):
         step()
@@ -288,10 +369,11 @@ def main():
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    # breakdown: the same K steps again with the library recording a CUDA event between its launches
-    # (events between launches defeat programmatic dependent launch, so the headline is taken above)
+    # breakdown: the same K local selects again with the library recording a CUDA event between its
+    # launches (events between launches defeat programmatic dependent launch, so the headline is
+    # taken above; for a split row this times the shard's local select only)
     for s_i in range(args.steps):
-        step(ev_sets[s_i][1])
+        at.select(xd, k, workspace=ws, out=(ov, oi), events=ev_sets[s_i][1], **sel_opts)
     torch.cuda.synchronize()
     clocks = sampler.stop()
     ms_local = t_start.elapsed_time(t_end) / args.steps
@@ -330,11 +412,12 @@ def main():
                         "peak_kind": peak_kind, "unit": "GB/s", "frac": ach / peak,
                         "peak_note": "MEASURED_PEAKS hbm_gbs is a copy (read+write) rate; a read-only "
                                      "stream can exceed it (frac slightly > 1)",
-                        "traffic": load_traffic(cfg, dom, n_launch),
+                        "traffic": load_traffic(plan_key(cfg, plan, sel_opts, args.dtype), dom),
+                        "traffic_plan": plan_key(cfg, plan, sel_opts, args.dtype),
                         "alg_bytes_per_launch": dom_alg, "launch_ms": float(per[dom])}
         whole = (in_bytes + out_bytes) / (select_ms * 1e-3) / 1e9
         result = {
-            "metric": "top-K elements/s and achieved HBM GB/s vs B200 peak (N=2^30,K=2^20; b=100)",
+            "metric": METRIC,
             "value": value, "unit": "elements/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": ms, "higher_is_better": True, "scaling": scaling, "vs_baseline": None,
             "dtype": args.dtype, "data": "synthetic",
@@ -387,6 +470,7 @@ def main():
             del xd, ws, ov, oi
             torch.cuda.empty_cache()
             result["extras"] = {name: extra_measure(name, dev) for name in ("c1", "c2", "c4")}
+            result["per_rank_proxies"] = per_rank_proxies(dev)
         print(json.dumps(result), flush=True)
     if world > 1:
         dist.barrier()
@@ -442,18 +526,107 @@ def plan_merge_launches(world, k):
     return at.describe(torch.float32, 1, world * k, k)["launches"]
 
 
-def load_traffic(cfg, q, n_launch):
-    """dram bytes (read + write) of launch q of a select, from the committed ncu launch list
-    (profiles/traffic_launches.json, written by tools/make_profiles.py from `ncu --metrics
-    dram__bytes_read.sum,dram__bytes_write.sum`): the second select of the list (warm), else the first."""
-    p = os.path.join(ROOT, "profiles", "traffic_launches.json")
+def plan_key(cfg, plan, sel_opts, dtype="f32"):
+    """Identifies a launch sequence: config, key type, engine, launch count and the window / bulk-copy
+    options (the same config runs different kernels under --window -1, --engine 4, ...)."""
+    return (f"{cfg}/{dtype}/engine{plan['engine']}/launches{plan['launches']}/window{sel_opts.get('window', 0)}"
+            f"/tma{sel_opts.get('tma', 0)}")
+
+
+def load_traffic(key, q):
+    """dram bytes (read + write) of launch q of the select identified by `key` (plan_key), from the
+    committed ncu launch list of the same plan (profiles/traffic.json, written by
+    tools/make_profiles.py from `ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum`): the
+    second select of the list (warm), else the first. None if that plan was not captured."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
     try:
         with open(p) as f:
-            d = json.load(f).get(cfg, {})
-        v = d.get(str(n_launch + q), d.get(str(q)))
-        return float(v) if v is not None else None
+            d = json.load(f).get(key)
+        if not d:
+            return None
+        n = d["launches_per_select"]
+        v = d["bytes"][n + q] if len(d["bytes"]) > n + q else d["bytes"][q]
+        return float(v)
     except Exception:
         return None
+
+
+def _timed(fn, steps, flush=None):
+    """Mean device time of fn() over `steps` calls, CUDA events around each call on the current
+    stream, L2 flushed (a 256 MB write) before each call when `flush` is given."""
+    import torch
+    tot = 0.0
+    for _ in range(steps):
+        if flush is not None:
+            flush.fill_(1)
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        fn()
+        e1.record()
+        e1.synchronize()
+        tot += e0.elapsed_time(e1)
+    return tot / steps
+
+
+def per_rank_proxies(dev, steps=100):
+    """What one rank of the 2/4/8-GPU runs does, measured on this one GPU: c2's
+    row shards (50 / 25 / 13 rows of 2^20 normal keys, K = 256; no collective) and c5's per-rank
+    work (the local select of a 2^30 uniform shard with K = 2^16, and the merge select over the
+    8 x 2^16 gathered candidates; the NCCL all-gather between them is not in these numbers)."""
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    peak, _ = hbm_peak()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    out = {}
+    c = CFG["c2"]
+    xh = host_keys("c2", c["n"], 50)
+    x50 = torch.from_numpy(xh).to(dev)
+    for rows in (50, 25, 13):
+        x = x50[:rows].contiguous()
+        ws = torch.empty(max(1, at.workspace_bytes(torch.float32, rows, c["n"], c["k"])), dtype=torch.uint8, device=dev)
+        o = (torch.empty((rows, c["k"]), dtype=torch.float32, device=dev),
+             torch.empty((rows, c["k"]), dtype=torch.int64, device=dev))
+        fn = lambda: at.select(x, c["k"], workspace=ws, out=o)
+        for _ in range(5):
+            fn()
+        ms = _timed(fn, steps, flush)
+        alg = rows * c["n"] * 4 + rows * c["k"] * 12
+        out[f"c2_rows{rows}"] = {"ms": ms, "elements_per_s": rows * c["n"] / (ms * 1e-3),
+                                 "roofline_ms": alg / (peak * 1e9) * 1e3,
+                                 "frac_of_peak": alg / (ms * 1e-3) / 1e9 / peak, "l2": "flushed"}
+    del x50
+    # c5 rank: local shard select (2^30 keys, global offset 0) + the 8 x 2^16 merge
+    n, k, world = 1 << 30, 1 << 16, 8
+    x = torch.from_numpy(host_keys("c5", n, 1)).to(dev).reshape(-1)
+    ws = torch.empty(max(1, at.lib().airtopk_workspace_bytes_shard(at.dtype_code(torch.float32), n, k)),
+                     dtype=torch.uint8, device=dev)
+    o = (torch.empty(k, dtype=torch.float32, device=dev), torch.empty(k, dtype=torch.int64, device=dev))
+    fn = lambda: at.select_shard(x, k, 0, (1 << 33), out=o, workspace=ws)
+    for _ in range(3):
+        fn()
+    ms = _timed(fn, 20)
+    alg = n * 4 + k * 12
+    out["c5_shard_select"] = {"ms": ms, "elements_per_s": n / (ms * 1e-3), "roofline_ms": alg / (peak * 1e9) * 1e3,
+                              "frac_of_peak": alg / (ms * 1e-3) / 1e9 / peak, "l2": "input > L2"}
+    del x
+    # merge input: 8 ranks' candidates = keys uniform on (0, 2^-14] (each shard's top 2^16 of 2^30
+    # uniform (0,1] keys lies there) with distinct global indices r * 2^30 + j * 2^14
+    m = world * k
+    gv = torch.from_numpy(gen.uniform_f32(gen.config_seed("c5") + 1, m) * np.float32(2.0 ** -14)).to(dev)
+    r = torch.arange(m, device=dev)
+    gi = (r // k) * (1 << 30) + (r % k) * (1 << 14)
+    bits = at.merge_idx_bits(1 << 33, world, k)
+    wsm = torch.empty(max(1, at.lib().airtopk_workspace_bytes_with_idx(at.dtype_code(torch.float32), m, k, bits)),
+                      dtype=torch.uint8, device=dev)
+    mo = (torch.empty(k, dtype=torch.float32, device=dev), torch.empty(k, dtype=torch.int64, device=dev))
+    fn = lambda: at.select_with_idx(gv, gi, k, bits, workspace=wsm, out=mo)
+    for _ in range(5):
+        fn()
+    ms = _timed(fn, steps, flush)
+    out["c5_merge_8x2^16"] = {"ms": ms, "elements_per_s": m / (ms * 1e-3), "l2": "flushed",
+                              "input": "8 x 2^16 keys uniform on (0, 2^-14], distinct global indices"}
+    return out
 
 
 def extra_measure(name, dev, steps=None, warmup=5):

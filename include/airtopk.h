@@ -41,8 +41,12 @@
  *   AIRTOPK_EINVAL     null pointer, batch < 1, len < 1, k < 1 or k > len (K in [1, N]);
  *   AIRTOPK_EDTYPE     unknown dtype;
  *   AIRTOPK_ENOSPACE   workspace smaller than airtopk_workspace_bytes(...);
- *   AIRTOPK_ECUDA      a CUDA launch/allocation failed (airtopk_last_cuda_error() has the code).
+ *   AIRTOPK_ECUDA      a CUDA launch/allocation failed (airtopk_last_cuda_error() has the code);
+ *   AIRTOPK_EDEVICE    (synchronous calls only: airtopk_select_host) the kernels flagged an
+ *                      inconsistency, e.g. duplicate in_idx values (see airtopk_options.status).
  * Faults inside kernels surface at the caller's next synchronisation, as with any CUDA library.
+ * Inconsistencies the kernels detect (more than K results or fewer, which only duplicate in_idx
+ * values can cause) are reported through the optional device word airtopk_options.status.
  * Nothing is written to the outputs when a status other than AIRTOPK_OK is returned.
  */
 #ifndef AIRTOPK_H_
@@ -63,8 +67,14 @@ typedef enum {
   AIRTOPK_EINVAL = 1,
   AIRTOPK_EDTYPE = 2,
   AIRTOPK_ENOSPACE = 3,
-  AIRTOPK_ECUDA = 4
+  AIRTOPK_ECUDA = 4,
+  AIRTOPK_EDEVICE = 5
 } airtopk_status;
+
+/* Bits OR-ed into *airtopk_options.status (device-detected inconsistencies; 0 = none). */
+#define AIRTOPK_ERR_OUTPUT_OVERFLOW 1u  /* more than K results in a row (duplicate in_idx values) */
+#define AIRTOPK_ERR_BUFFER_OVERFLOW 2u  /* a candidate buffer overflowed outside the window pass */
+#define AIRTOPK_ERR_COUNT 4u            /* histogram total != candidates, or fewer than K results */
 
 typedef enum {
   AIRTOPK_F32 = 0,  /* IEEE binary32, r = 32 bits: 3 radix passes of 11/11/10 bits */
@@ -111,6 +121,9 @@ typedef struct {
                            -1 = register loads. */
   int32_t early_stop;   /* early stopping: 0 = on (default), -1 = off (the Fig. 10 ablation:
                            the passes continue after K == C; results identical). */
+  uint32_t* status;     /* optional DEVICE word: after the select the library ORs every row's
+                           AIRTOPK_ERR_* flags into it (one extra tiny launch; the caller zeroes it and
+                           reads it after synchronising). NULL = not collected. Radix engines only. */
 } airtopk_options;
 
 #define AIRTOPK_TRACE_MAX_PASSES 16
@@ -154,6 +167,33 @@ airtopk_status airtopk_select_with_idx(const void* keys, const int64_t* in_idx, 
                                        airtopk_dtype dtype, int64_t len, int64_t k, int select_min,
                                        void* out_vals, int64_t* out_idx, void* workspace,
                                        size_t workspace_bytes, airtopk_stream_t stream);
+
+/* Same with options (alpha, engine 1/2, status word, events, ...). */
+airtopk_status airtopk_select_with_idx_ex(const void* keys, const int64_t* in_idx, int idx_bits,
+                                          airtopk_dtype dtype, int64_t len, int64_t k, int select_min,
+                                          void* out_vals, int64_t* out_idx, void* workspace,
+                                          size_t workspace_bytes, airtopk_stream_t stream,
+                                          const airtopk_options* opt);
+
+/* Multi-GPU split row ("top 0.1% ... across workers").
+ * One row of total_len keys is split into contiguous shards, one per rank. Each rank calls
+ * airtopk_select_shard on its shard (len keys starting at global index shard_offset): it writes
+ * exactly k entries — the min(k, len) smallest (largest) keys of the shard with GLOBAL indices
+ * (local index + shard_offset; ties by lowest index, P:78 reading), and, when len < k, k - len pad
+ * entries whose key sorts after every key (the maximum code) with indices pad_base + j, j < k - len.
+ * The caller picks pad_base = total_len + rank * k so pad indices never collide. out_vals [k] of
+ * the key type, out_idx [k] int64, device memory; the k entries of every rank are gathered
+ * (one NCCL all-gather, or peer stores) into [world * k] arrays, and airtopk_select_with_idx with
+ * idx_bits = airtopk_merge_idx_bits(total_len, world, k) gives the global top-k on every rank
+ * (exact: a global top-k element has < k predecessors in (code, index) order, hence < k in its own
+ * shard). Workspace: airtopk_workspace_bytes_shard(dtype, len, k) bytes, 256-aligned, device. */
+size_t airtopk_workspace_bytes_shard(airtopk_dtype dtype, int64_t len, int64_t k);
+airtopk_status airtopk_select_shard(const void* keys, airtopk_dtype dtype, int64_t len, int64_t k,
+                                    int select_min, int64_t shard_offset, int64_t pad_base,
+                                    void* out_vals, int64_t* out_idx, void* workspace,
+                                    size_t workspace_bytes, airtopk_stream_t stream);
+/* Index width of the merge select: bits of total_len + world * k - 1 (0 on invalid arguments). */
+int airtopk_merge_idx_bits(int64_t total_len, int world, int64_t k);
 
 /* End-to-end convenience with HOST buffers: copies keys host->device, selects, copies the results
  * device->host and SYNCHRONISES `stream` before returning. Pinned (page-locked) host memory gives

@@ -25,10 +25,11 @@ DT_NAMES = {"f32": 0, "f16": 1, "bf16": 2, "f64": 3, "u32": 4}
 
 
 def build(force: bool = False) -> str:
-    """Compile the oracle (plain C++17, -O2, no OpenMP: the timed baseline is single-core)."""
+    """Compile the oracle (plain C++17, -O2; OpenMP only in oracle_topk_nth_mt, the all-cores
+    CPU baseline variant — every other function is single-threaded)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["g++", "-std=c++17", "-O2", "-fPIC", "-shared", _SRC, "-o", tmp])
+        subprocess.check_call(["g++", "-std=c++17", "-O2", "-fopenmp", "-fPIC", "-shared", _SRC, "-o", tmp])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -43,6 +44,8 @@ def _L():
             f = getattr(lib, name)
             f.argtypes = [ci, vp, i64, i64, i64, ci, vp, vp]
             f.restype = ci
+        lib.oracle_topk_nth_mt.argtypes = [ci, vp, i64, i64, i64, ci, vp, vp, ctypes.POINTER(ci)]
+        lib.oracle_topk_nth_mt.restype = ci
         lib.oracle_topk_with_idx.argtypes = [ci, vp, vp, i64, i64, ci, vp, vp]
         lib.oracle_topk_with_idx.restype = ci
         lib.oracle_codes.argtypes = [ci, vp, i64, ci, vp]
@@ -89,6 +92,20 @@ def topk_sort(keys, k, select_min=True, dt=None):
 
 def topk_nth(keys, k, select_min=True, dt=None):
     return _run("oracle_topk_nth", keys, k, select_min, dt)
+
+
+def topk_nth_mt(keys, k, select_min=True, dt=None):
+    """All-cores variant (OpenMP chunks + candidate merge). Returns (values, indices, threads)."""
+    keys, dt = _prep(keys, dt)
+    batch, n = keys.shape
+    vals = np.empty((batch, k), dtype=keys.dtype)
+    idx = np.empty((batch, k), dtype=np.int64)
+    th = ctypes.c_int(0)
+    rc = _L().oracle_topk_nth_mt(dt, keys.ctypes.data, batch, n, k, int(bool(select_min)),
+                                 vals.ctypes.data, idx.ctypes.data, ctypes.byref(th))
+    if rc != 0:
+        raise ValueError(f"oracle_topk_nth_mt failed rc={rc}")
+    return vals, idx, int(th.value)
 
 
 def topk_brute(keys, k, select_min=True, dt=None):

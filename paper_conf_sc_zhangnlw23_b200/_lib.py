@@ -10,9 +10,10 @@ import os
 _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("AIRTOPK_LIB", os.path.join(_PKG, "libairtopk.so"))
 
-OK, EINVAL, EDTYPE, ENOSPACE, ECUDA = 0, 1, 2, 3, 4
+OK, EINVAL, EDTYPE, ENOSPACE, ECUDA, EDEVICE = 0, 1, 2, 3, 4, 5
+ERR_OUTPUT_OVERFLOW, ERR_BUFFER_OVERFLOW, ERR_COUNT = 1, 2, 4
 F32, F16, BF16, F64, U32 = 0, 1, 2, 3, 4
-ENGINE_AUTO, ENGINE_GRID, ENGINE_CLUSTER, ENGINE_GRIDSELECT = 0, 1, 2, 4
+ENGINE_AUTO, ENGINE_GRID, ENGINE_CLUSTER, ENGINE_GRIDSELECT, ENGINE_BATCH = 0, 1, 2, 4, 5
 TRACE_MAX_PASSES = 16
 TRACE_FIELDS = ("width", "src_L", "stored", "j", "K", "C", "Cp", "emitted", "early_stop", "read")
 
@@ -22,7 +23,8 @@ EXPORTS = (
     "airtopk_select_f32", "airtopk_select_f16", "airtopk_select_bf16", "airtopk_select_f64",
     "airtopk_select_u32", "airtopk_workspace_bytes_with_idx", "airtopk_select_with_idx",
     "airtopk_select_host", "airtopk_status_str", "airtopk_last_cuda_error", "airtopk_version",
-    "airtopk_describe",
+    "airtopk_describe", "airtopk_select_with_idx_ex", "airtopk_workspace_bytes_shard", "airtopk_select_shard",
+    "airtopk_merge_idx_bits",
 )
 
 
@@ -38,6 +40,7 @@ class Options(ctypes.Structure):
         ("window", ctypes.c_int32),
         ("tma", ctypes.c_int32),
         ("early_stop", ctypes.c_int32),
+        ("status", ctypes.c_void_p),
     ]
 
 
@@ -85,6 +88,14 @@ def load(path: str = LIB_PATH):
     lib.airtopk_workspace_bytes_with_idx.restype = sz
     lib.airtopk_select_with_idx.argtypes = [vp, vp, ci, ci, i64, i64, ci, vp, vp, vp, sz, vp]
     lib.airtopk_select_with_idx.restype = ci
+    lib.airtopk_select_with_idx_ex.argtypes = [vp, vp, ci, ci, i64, i64, ci, vp, vp, vp, sz, vp, ctypes.POINTER(Options)]
+    lib.airtopk_select_with_idx_ex.restype = ci
+    lib.airtopk_workspace_bytes_shard.argtypes = [ci, i64, i64]
+    lib.airtopk_workspace_bytes_shard.restype = sz
+    lib.airtopk_select_shard.argtypes = [vp, ci, i64, i64, ci, i64, i64, vp, vp, vp, sz, vp]
+    lib.airtopk_select_shard.restype = ci
+    lib.airtopk_merge_idx_bits.argtypes = [i64, ci, i64]
+    lib.airtopk_merge_idx_bits.restype = ci
     lib.airtopk_select_host.argtypes = [vp, ci, i64, i64, i64, ci, vp, vp, vp]
     lib.airtopk_select_host.restype = ci
     lib.airtopk_status_str.argtypes = [ci]

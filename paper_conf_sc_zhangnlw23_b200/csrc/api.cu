@@ -5,8 +5,13 @@
 // stream (the iteration-fused property: the CPU only launches kernels, P:50/P:142/P:158).
 #include <algorithm>
 #include <cstdlib>
+#include <mutex>
+#include <set>
+#include <tuple>
 #include <cmath>
 #include <cstring>
+
+#include <nvtx3/nvToolsExt.h>
 
 #include "../../include/airtopk.h"
 #include "device.cuh"
@@ -26,6 +31,26 @@ int bits_needed(uint64_t v) {  // number of bits to represent v (0 for v == 0)
 }
 
 }  // namespace
+
+cudaError_t func_attr(const void* f, cudaFuncAttribute attr, int value) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  using Key = std::tuple<const void*, int, int, int>;
+  static std::mutex mu;
+  static std::set<Key> done;
+  const Key key{f, dev, (int)attr, value};
+  {
+    std::lock_guard<std::mutex> g(mu);
+    if (done.count(key)) return cudaSuccess;
+  }
+  e = cudaFuncSetAttribute(f, attr, value);
+  if (e == cudaSuccess) {
+    std::lock_guard<std::mutex> g(mu);
+    done.insert(key);
+  }
+  return e;
+}
 
 int num_sms() {
   static thread_local int dev_cached = -1, sms_cached = 148;
@@ -188,9 +213,17 @@ static airtopk_status fail_cuda(cudaError_t e) {
   return AIRTOPK_ECUDA;
 }
 
+// NVTX range around everything one select enqueues (the paper's per-call measurement unit, P:210;
+// lets nsys / ncu --nvtx delimit a select). No cost without an attached tool.
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+
 static airtopk_status run(const SelectArgs& a, void* ws, size_t ws_bytes, cudaStream_t s) {
   airtopk_status st = validate(a);
   if (st != AIRTOPK_OK) return st;
+  NvtxRange nvtx(a.in_idx ? "airtopk_select_with_idx" : "airtopk_select");
   Plan p = make_plan(a);
   if (p.engine == 3) {
     cudaError_t e = run_trivial(a, s);
@@ -205,6 +238,7 @@ static airtopk_status run(const SelectArgs& a, void* ws, size_t ws_bytes, cudaSt
   choose_launch(a, p);
   if (p.engine == 2 && (p.csize < 1 || p.csize > 16 || (p.csize & (p.csize - 1)))) return AIRTOPK_EINVAL;
   cudaError_t e = (p.engine == 2) ? run_cluster(a, p, ws, s) : run_grid(a, p, ws, s);
+  if (e == cudaSuccess && a.status) e = collect_status(a, p, ws, s);
   return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
 }
 
@@ -230,6 +264,7 @@ static SelectArgs make_args(const void* keys, int dt, int64_t batch, int64_t len
     a.window = opt->window;
     a.tma = opt->tma;
     a.early_stop = opt->early_stop;
+    a.status = opt->status;
   }
   if (a.alpha == 0) a.alpha = 128;
   return a;
@@ -330,6 +365,7 @@ airtopk_status airtopk_select_host(const void* h_keys, airtopk_dtype dtype, int6
   Plan p = make_plan(a);
   const size_t ws_b = p.engine == 3 ? 0 : p.bytes;
   const size_t o1 = align_up(in_b, 256), o2 = o1 + align_up(ov_b, 256), o3 = o2 + align_up(oi_b, 256);
+  const size_t o4 = o3 + align_up(ws_b, 256);  // the device status word
   // device staging cached per thread and device (this call synchronises before returning, so the
   // next call on this thread may reuse it); grows on demand, released at thread exit
   struct Staging {
@@ -342,34 +378,84 @@ airtopk_status airtopk_select_host(const void* h_keys, airtopk_dtype dtype, int6
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return fail_cuda(e);
-  if (stg.dev != dev || stg.bytes < o3 + ws_b) {
+  if (stg.dev != dev || stg.bytes < o4 + 256) {
     if (stg.ptr) {
       cudaStreamSynchronize(s);
       cudaFree(stg.ptr);
       stg.ptr = nullptr;
     }
-    if ((e = cudaMalloc((void**)&stg.ptr, o3 + ws_b)) != cudaSuccess) {
+    if ((e = cudaMalloc((void**)&stg.ptr, o4 + 256)) != cudaSuccess) {
       stg.bytes = 0;
       return fail_cuda(e);
     }
-    stg.bytes = o3 + ws_b;
+    stg.bytes = o4 + 256;
     stg.dev = dev;
   }
   char* d = stg.ptr;
+  unsigned* dstatus = (unsigned*)(d + o4);
   airtopk_status st = AIRTOPK_OK;
   if ((e = cudaMemcpyAsync(d, h_keys, in_b, cudaMemcpyHostToDevice, s)) != cudaSuccess) st = fail_cuda(e);
+  if (st == AIRTOPK_OK && (e = cudaMemsetAsync(dstatus, 0, sizeof(unsigned), s)) != cudaSuccess) st = fail_cuda(e);
   if (st == AIRTOPK_OK) {
     a.keys = d;
     a.out_vals = d + o1;
     a.out_idx = (int64_t*)(d + o2);
+    a.status = dstatus;
     st = run(a, ws_b ? d + o3 : nullptr, ws_b, s);
   }
   if (st == AIRTOPK_OK && (e = cudaMemcpyAsync(h_out_vals, d + o1, ov_b, cudaMemcpyDeviceToHost, s)) != cudaSuccess)
     st = fail_cuda(e);
   if (st == AIRTOPK_OK && (e = cudaMemcpyAsync(h_out_idx, d + o2, oi_b, cudaMemcpyDeviceToHost, s)) != cudaSuccess)
     st = fail_cuda(e);
+  unsigned hstatus = 0;
+  if (st == AIRTOPK_OK && (e = cudaMemcpyAsync(&hstatus, dstatus, sizeof(unsigned), cudaMemcpyDeviceToHost, s)) !=
+                              cudaSuccess)
+    st = fail_cuda(e);
   if ((e = cudaStreamSynchronize(s)) != cudaSuccess && st == AIRTOPK_OK) st = fail_cuda(e);
+  if (st == AIRTOPK_OK && hstatus != 0) st = AIRTOPK_EDEVICE;
   return st;
+}
+
+airtopk_status airtopk_select_with_idx_ex(const void* keys, const int64_t* in_idx, int idx_bits, airtopk_dtype dtype,
+                                          int64_t len, int64_t k, int select_min, void* out_vals, int64_t* out_idx,
+                                          void* workspace, size_t workspace_bytes, airtopk_stream_t stream,
+                                          const airtopk_options* opt) {
+  if (!in_idx) return AIRTOPK_EINVAL;
+  SelectArgs a = make_args(keys, (int)dtype, 1, len, k, select_min, out_vals, out_idx, opt);
+  if (a.engine == 4) return AIRTOPK_EINVAL;
+  a.in_idx = in_idx;
+  a.idx_bits = idx_bits;
+  a.window = 0;
+  return run(a, workspace, workspace_bytes, (cudaStream_t)stream);
+}
+
+int airtopk_merge_idx_bits(int64_t total_len, int world, int64_t k) {
+  if (total_len < 1 || world < 1 || k < 1) return 0;
+  // real global indices < total_len; pad indices total_len + r*k + j < total_len + world*k
+  const int b = bits_needed((uint64_t)(total_len + (int64_t)world * k - 1));
+  return b < 1 ? 1 : b;
+}
+
+size_t airtopk_workspace_bytes_shard(airtopk_dtype dtype, int64_t len, int64_t k) {
+  if (len < 1 || k < 1) return 0;
+  return airtopk_workspace_bytes(dtype, 1, len, std::min(k, len));
+}
+
+airtopk_status airtopk_select_shard(const void* keys, airtopk_dtype dtype, int64_t len, int64_t k, int select_min,
+                                    int64_t shard_offset, int64_t pad_base, void* out_vals, int64_t* out_idx,
+                                    void* workspace, size_t workspace_bytes, airtopk_stream_t stream) {
+  if (!keys || !out_vals || !out_idx) return AIRTOPK_EINVAL;
+  if (!valid_kind((int)dtype)) return AIRTOPK_EDTYPE;
+  if (len < 1 || k < 1 || shard_offset < 0 || pad_base < 0) return AIRTOPK_EINVAL;
+  NvtxRange nvtx("airtopk_select_shard");
+  const int64_t kk = std::min(k, len);
+  SelectArgs a = make_args(keys, (int)dtype, 1, len, kk, select_min, out_vals, out_idx, nullptr);
+  a.idx_off = shard_offset;
+  airtopk_status st = run(a, workspace, workspace_bytes, (cudaStream_t)stream);
+  if (st != AIRTOPK_OK || kk == k) return st;
+  cudaError_t e = run_pad(a.kind, a.sel_min, (char*)out_vals + (size_t)kk * key_bytes(a.kind), out_idx + kk, k - kk,
+                          pad_base, (cudaStream_t)stream);
+  return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
 }
 
 airtopk_status airtopk_describe(airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k,
@@ -401,6 +487,7 @@ const char* airtopk_status_str(airtopk_status s) {
     case AIRTOPK_EDTYPE: return "AIRTOPK_EDTYPE: unknown dtype";
     case AIRTOPK_ENOSPACE: return "AIRTOPK_ENOSPACE: workspace too small";
     case AIRTOPK_ECUDA: return "AIRTOPK_ECUDA: CUDA error (see airtopk_last_cuda_error)";
+    case AIRTOPK_EDEVICE: return "AIRTOPK_EDEVICE: the kernels detected inconsistent input (e.g. duplicate in_idx values)";
   }
   return "AIRTOPK: unknown status";
 }

@@ -23,6 +23,8 @@ struct SelectArgs {
   int window = 0;                   // sample-guided window: 0 auto, 1 on, -1 off
   int tma = 0;                      // bulk-copy streaming: 0 auto, 1 on, -1 off
   int early_stop = 0;               // 0 on, -1 off (ablation)
+  int64_t idx_off = 0;              // added to every output index (airtopk_select_shard)
+  unsigned* status = nullptr;       // optional device word: row error flags OR-ed in after the select
   int64_t* trace = nullptr;
   void* const* events = nullptr;    // optional cudaEvent_t[n_events] recorded around launches
   int n_events = 0;
@@ -48,6 +50,14 @@ struct Plan {
   size_t off_state, off_hist, off_bcode, off_bidx, off_samp, bytes;
 };
 
+// cudaFuncSetAttribute once per (kernel, current device, attribute, value): the runtime applies
+// function attributes per device, so a process selecting on several GPUs sets them on each.
+cudaError_t func_attr(const void* func, cudaFuncAttribute attr, int value);
+template <typename F>
+cudaError_t func_attr(F* func, cudaFuncAttribute attr, int value) {
+  return func_attr(reinterpret_cast<const void*>(func), attr, value);
+}
+
 int key_bits(int kind);
 int num_sms();  // SMs of the current device (cached per thread)
 int key_bytes(int kind);
@@ -55,6 +65,11 @@ Plan make_plan(const SelectArgs& a);
 cudaError_t run_grid(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 cudaError_t run_cluster(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 cudaError_t run_trivial(const SelectArgs& a, cudaStream_t s);
+// K entries that sort last in the selection order (multi-GPU shard shorter than K): value bits of the
+// maximum code, indices pad_base + j
+cudaError_t run_pad(int kind, int sel_min, void* vals, int64_t* idx, int64_t n, int64_t pad_base, cudaStream_t s);
+// OR the error flags of every row state of a grid / cluster engine workspace into *a.status
+cudaError_t collect_status(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 int grid_blocks_per_sm(const SelectArgs& a, int idx64);
 // GridSelect: keys of <= 32 bits, len < 2^32, K <= 256
 bool gridselect_supported(const SelectArgs& a);

@@ -45,6 +45,7 @@ struct ClusterParams {
   int64_t cap_rule, cap_alloc;
   int nclusters;
   int early_stop;  // 0 on, -1 off (ablation)
+  int64_t idx_off; // added to every output index (airtopk_select_shard)
   int tail;      // 1: continue rows after the grid engine's window pass
   int tail_q;    // tail mode: the grid engine ran passes q < tail_q after the window pass
   int timing_stride;  // int64 slots per CTA in `timing` (8; 24 with the merge-phase stamps, debug)
@@ -172,6 +173,7 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
       c.nbuf = (src1 > 0) ? __ldcg(&st->buf_count[islot]) : 0ull;
       c.ov = (U*)p.out_vals + row * p.k;
       c.oi = p.out_idx + row * p.k;
+      c.ioff = p.idx_off;
       c.outc = &st->out_count;
       c.kk = kk;
       c.bco = (U*)p.bcode + ((size_t)sslot * p.batch + row) * p.cap_alloc;
@@ -280,8 +282,8 @@ template <int KIND, typename IdxT, bool HASIDX>
 cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t s, int tail) {
   auto kern = cluster_kernel<KIND, IdxT, HASIDX>;
   constexpr size_t smem = (size_t)kHistSlots * 4;
-  static const cudaError_t attr1 = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  static const cudaError_t attr2 = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+  const cudaError_t attr1 = func_attr(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  const cudaError_t attr2 = func_attr(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
   if (attr1 != cudaSuccess) return attr1;
   if (attr2 != cudaSuccess) return attr2;
   char* base = (char*)ws;
@@ -304,6 +306,7 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   p.cap_alloc = pl.cap_alloc;
   p.tail = tail;
   p.early_stop = a.early_stop;
+  p.idx_off = a.idx_off;
   p.tail_q = pl.tail_q;
   p.timing = a.trace;  // cluster engine: the trace buffer receives per-CTA timing instead
   p.timing_stride = getenv("AIRTOPK_CLUSTER_TIMING") ? 24 : 8;

@@ -22,10 +22,10 @@ extern template cudaError_t launch_cluster_kind<K_U32>(const SelectArgs&, const 
 
 // K == N ("a trivial case"): every element is a result, in index order.
 template <typename U>
-__global__ void trivial_kernel(const U* keys, int64_t total, U* ov, int64_t* oi, int64_t len) {
+__global__ void trivial_kernel(const U* keys, int64_t total, U* ov, int64_t* oi, int64_t len, int64_t ioff) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     ov[i] = keys[i];
-    oi[i] = i % len;
+    oi[i] = i % len + ioff;
   }
 }
 
@@ -64,6 +64,7 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t
   gp.samp = base + pl.off_samp;
   gp.nsms = num_sms();
   gp.early_stop = a.early_stop;
+  gp.idx_off = a.idx_off;
   {
     static const char* env2 = getenv("AIRTOPK_SMALL_FINISH");  // A/B knob (0 = off)
     gp.small_finish = env2 ? std::min(atoi(env2), kSmallFinish) : kSmallFinish;
@@ -89,14 +90,50 @@ cudaError_t run_cluster(const SelectArgs& a, const Plan& pl, void* ws, cudaStrea
   return cudaErrorInvalidValue;
 }
 
+template <int KIND>
+__global__ void pad_kernel(typename KT<KIND>::U* ov, int64_t* oi, int64_t n, int64_t pad_base, int sel_min) {
+  using U = typename KT<KIND>::U;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    ov[i] = from_code<KIND>((U)~(U)0, sel_min != 0);  // the largest code: sorts after every key
+    oi[i] = pad_base + i;
+  }
+}
+
+cudaError_t run_pad(int kind, int sel_min, void* vals, int64_t* idx, int64_t n, int64_t pad_base, cudaStream_t s) {
+  const unsigned blocks = (unsigned)std::min<int64_t>((n + 255) / 256, 1024);
+  switch (kind) {
+    case K_F32: pad_kernel<K_F32><<<blocks, 256, 0, s>>>((uint32_t*)vals, idx, n, pad_base, sel_min); break;
+    case K_F16: pad_kernel<K_F16><<<blocks, 256, 0, s>>>((uint16_t*)vals, idx, n, pad_base, sel_min); break;
+    case K_BF16: pad_kernel<K_BF16><<<blocks, 256, 0, s>>>((uint16_t*)vals, idx, n, pad_base, sel_min); break;
+    case K_F64: pad_kernel<K_F64><<<blocks, 256, 0, s>>>((uint64_t*)vals, idx, n, pad_base, sel_min); break;
+    case K_U32: pad_kernel<K_U32><<<blocks, 256, 0, s>>>((uint32_t*)vals, idx, n, pad_base, sel_min); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+__global__ void status_kernel(const RowState* st, int64_t batch, unsigned* status) {
+  unsigned e = 0;
+  for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < batch; r += (int64_t)gridDim.x * blockDim.x)
+    e |= st[r].error;
+  e = __reduce_or_sync(kFull, e);
+  if ((threadIdx.x & 31) == 0 && e) atomicOr(status, e);
+}
+
+cudaError_t collect_status(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s) {
+  const unsigned blocks = (unsigned)std::min<int64_t>((a.batch + 255) / 256, 148);
+  status_kernel<<<blocks, 256, 0, s>>>((const RowState*)((char*)ws + p.off_state), a.batch, a.status);
+  return cudaGetLastError();
+}
+
 cudaError_t run_trivial(const SelectArgs& a, cudaStream_t s) {
   const int64_t total = a.batch * a.len;
   const int threads = 256;
   const long long blocks = std::min<long long>((total + threads - 1) / threads, 148LL * 16);
   switch (key_bytes(a.kind)) {
-    case 2: trivial_kernel<uint16_t><<<(unsigned)blocks, threads, 0, s>>>((const uint16_t*)a.keys, total, (uint16_t*)a.out_vals, a.out_idx, a.len); break;
-    case 4: trivial_kernel<uint32_t><<<(unsigned)blocks, threads, 0, s>>>((const uint32_t*)a.keys, total, (uint32_t*)a.out_vals, a.out_idx, a.len); break;
-    default: trivial_kernel<uint64_t><<<(unsigned)blocks, threads, 0, s>>>((const uint64_t*)a.keys, total, (uint64_t*)a.out_vals, a.out_idx, a.len); break;
+    case 2: trivial_kernel<uint16_t><<<(unsigned)blocks, threads, 0, s>>>((const uint16_t*)a.keys, total, (uint16_t*)a.out_vals, a.out_idx, a.len, a.idx_off); break;
+    case 4: trivial_kernel<uint32_t><<<(unsigned)blocks, threads, 0, s>>>((const uint32_t*)a.keys, total, (uint32_t*)a.out_vals, a.out_idx, a.len, a.idx_off); break;
+    default: trivial_kernel<uint64_t><<<(unsigned)blocks, threads, 0, s>>>((const uint64_t*)a.keys, total, (uint64_t*)a.out_vals, a.out_idx, a.len, a.idx_off); break;
   }
   return cudaGetLastError();
 }

@@ -67,6 +67,7 @@ struct GridParams {
   int nsms;    // SMs of the device
   int small_finish;  // a buffer-source pass over <= this many entries finishes the row in one CTA
   int early_stop;   // 0 on, -1 off (ablation)
+  int64_t idx_off;  // added to every output index (airtopk_select_shard)
 };
 
 constexpr int kBlock = 512;
@@ -180,6 +181,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.nbuf = (src1 > 0) ? st->buf_count[islot] : 0ull;
   c.ov = (U*)p.out_vals + row * p.k;
   c.oi = p.out_idx + row * p.k;
+  c.ioff = p.idx_off;
   c.outc = &st->out_count;
   c.kk = (unsigned long long)p.k;
   c.bco = (U*)p.bcode + ((size_t)sslot * p.batch + row) * p.cap_alloc;
@@ -704,8 +706,8 @@ constexpr size_t hist_smem_bytes() {
 template <int KIND, typename IdxT, int DF, int DH, bool HASIDX, bool TMA>
 cudaError_t launch_one(const GridParams& gp, unsigned grid, int q, int redo, cudaStream_t s) {
   constexpr size_t smem = hist_smem_bytes<KIND, IdxT, DF, DH, TMA>();
-  static const cudaError_t attr = cudaFuncSetAttribute(pass_kernel<KIND, IdxT, DF, DH, HASIDX, TMA>,
-                                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  const cudaError_t attr = func_attr(pass_kernel<KIND, IdxT, DF, DH, HASIDX, TMA>,
+                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (attr != cudaSuccess) return attr;
   return launch_pdl(pass_kernel<KIND, IdxT, DF, DH, HASIDX, TMA>, dim3(grid), dim3(kBlock), smem, s, gp, q, redo);
 }
@@ -731,10 +733,10 @@ cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, c
   if (nsamp > 0) {  // sample-guided window: sample, window pass (= pass 0 + filter), pass 0 over the window
     using W = std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long, unsigned>;
     const size_t smem = (size_t)kMaxSamples * 4;  // 8-byte keys: nsamp <= kMaxSamples / 2
-    static const cudaError_t attr =
-        cudaFuncSetAttribute(sample_kernel<KIND, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    static const cudaError_t attr1 =
-        cudaFuncSetAttribute(sample_kernel<KIND, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const cudaError_t attr =
+        func_attr(sample_kernel<KIND, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const cudaError_t attr1 =
+        func_attr(sample_kernel<KIND, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (attr != cudaSuccess) return attr;
     if (attr1 != cudaSuccess) return attr1;
     // CTAs per row: enough to spread a few rows' scattered loads over the SMs; one per row for

@@ -100,7 +100,7 @@ template <int KIND, typename IdxT>
 __device__ __noinline__ void wq_write(const WarpQ<typename KT<KIND>::U, IdxT>* wq, int n, unsigned long long br,
                                       unsigned long long bc, typename KT<KIND>::U* ov, int64_t* oi,
                                       unsigned long long kk, typename KT<KIND>::U* bco, IdxT* bio,
-                                      unsigned long long capa, bool sel_min, unsigned* err) {
+                                      unsigned long long capa, bool sel_min, unsigned* err, int64_t ioff) {
   const int lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
   for (int j0 = 0; j0 < n; j0 += 32) {
@@ -111,7 +111,7 @@ __device__ __noinline__ void wq_write(const WarpQ<typename KT<KIND>::U, IdxT>* w
       const unsigned long long pos = br + __popc(mr & lt);
       if (pos < kk) {
         ov[pos] = from_code<KIND>(wq->code[j], sel_min);
-        oi[pos] = (int64_t)wq->idx[j];
+        oi[pos] = (int64_t)wq->idx[j] + ioff;
       } else {
         *err |= 1u;
       }
@@ -149,14 +149,14 @@ template <int KIND, typename IdxT>
 __device__ __forceinline__ void wq_flush(const WarpQ<typename KT<KIND>::U, IdxT>* wq, int n, unsigned long long* outc,
                                       unsigned long long* bufc, typename KT<KIND>::U* ov, int64_t* oi,
                                       unsigned long long kk, typename KT<KIND>::U* bco, IdxT* bio,
-                                      unsigned long long capa, bool sel_min, unsigned* err) {
+                                      unsigned long long capa, bool sel_min, unsigned* err, int64_t ioff) {
   const int lane = threadIdx.x & 31;
   const unsigned cnt = wq_counts(wq, n);
   unsigned long long b = 0;
   if (lane == 0 && (cnt & 0xffffu)) b = atomicAdd(outc, (unsigned long long)(cnt & 0xffffu));
   if (lane == 1 && (cnt >> 16)) b = atomicAdd(bufc, (unsigned long long)(cnt >> 16));
   const unsigned long long br = __shfl_sync(kFull, b, 0), bc = __shfl_sync(kFull, b, 1);
-  wq_write<KIND, IdxT>(wq, n, br, bc, ov, oi, kk, bco, bio, capa, sel_min, err);
+  wq_write<KIND, IdxT>(wq, n, br, bc, ov, oi, kk, bco, bio, capa, sel_min, err, ioff);
 }
 
 // Everything one pass of one row needs (built by the engine from its copy of the row state).
@@ -178,6 +178,7 @@ struct PassCtx {
   // results
   U* ov;
   int64_t* oi;
+  int64_t ioff;     // added to every output index (multi-GPU shard: global index = local + offset)
   unsigned long long* outc;
   unsigned long long kk;
   // candidates
@@ -328,7 +329,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
   int qcnt = 0;
   auto flush_full = [&]() {
     __syncwarp();
-    wq_flush<KIND, IdxT>(wq, qcnt, c.outc, c.bufc, c.ov, c.oi, c.kk, c.bco, c.bio, c.capa, sel_min, c.err);
+    wq_flush<KIND, IdxT>(wq, qcnt, c.outc, c.bufc, c.ov, c.oi, c.kk, c.bco, c.bio, c.capa, sel_min, c.err, c.ioff);
     qcnt = 0;
     __syncwarp();
   };
@@ -732,7 +733,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
     __syncthreads();
     if (qcnt)
       wq_write<KIND, IdxT>(wq, qcnt, s_base[0][warp], s_base[1][warp], c.ov, c.oi, c.kk, c.bco, c.bio, c.capa,
-                           sel_min, c.err);
+                           sel_min, c.err, c.ioff);
   }
   if constexpr (DF == 3) {  // one atomic per warp: window-member extremes (the tail skips digits
                             // on which all members agree)
@@ -780,7 +781,7 @@ __device__ void small_finish(const PassCtx<typename KT<KIND>::U, IdxT>& c, unsig
       const unsigned long long pos = b + __popc(m & lanemask_lt());
       if (pos < c.kk) {
         c.ov[pos] = from_code<KIND>(code, c.sel_min);
-        c.oi[pos] = (int64_t)idx;
+        c.oi[pos] = (int64_t)idx + c.ioff;
       } else {
         atomicOr(c.err, 1u);
       }

@@ -23,9 +23,20 @@ def _free_port():
     return p
 
 
-def _oracle_select(t, k, largest):
-    v, i = oracle.topk_sort(t.numpy().reshape(1, -1), k, select_min=not largest)
-    return torch.from_numpy(v[0]), torch.from_numpy(i[0])
+def _oracle_shard(t, k, off, pad_base, largest, out):
+    """The contract of airtopk_select_shard, on the CPU oracle: the shard's top min(k, n) with
+    global indices, then pads (keys that sort last, indices pad_base + j)."""
+    from paper_conf_sc_zhangnlw23_b200 import dist as atd
+    x = t.numpy().reshape(1, -1)
+    kk = min(k, x.shape[1])
+    v, i = oracle.topk_sort(x, kk, select_min=not largest)
+    ov, oi = out
+    ov[:kk] = torch.from_numpy(v[0])
+    oi[:kk] = torch.from_numpy(i[0]) + off
+    if kk < k:
+        bits = atd.pad_bits(t.dtype, largest)
+        ov[kk:] = torch.from_numpy(np.full(k - kk, bits, dtype=np.uint32).view(np.float32))
+        oi[kk:] = pad_base + torch.arange(k - kk)
 
 
 def _oracle_merge(gv, gi, k, idx_bits, largest):
@@ -42,7 +53,7 @@ def _one(rank, world, case):
         lo, hi = int(bounds[rank]), int(bounds[rank + 1])
         x = gen.keys(case["dist"], 7, n_total, m_bits=case.get("m", 20))
         v, i = atd.select_split_row(torch.from_numpy(x[lo:hi].copy()), k, total_len=n_total, shard_offset=lo,
-                                    largest=largest, select_fn=_oracle_select, merge_fn=_oracle_merge)
+                                    largest=largest, shard_fn=_oracle_shard, merge_fn=_oracle_merge)
         rv, ri = oracle.topk_sort(x, k, select_min=not largest)
         ok = np.array_equal(np.sort(i.numpy()), np.sort(ri[0]))
         ok &= np.array_equal(np.sort(v.numpy().view(np.uint32)), np.sort(rv[0].view(np.uint32)))

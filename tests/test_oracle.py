@@ -138,8 +138,20 @@ def test_three_oracles_agree(dtn, n, kfrac, seed, pool, select_min, batch):
     a = oracle.topk_sort(raw, k, select_min, dt=dt)
     b = oracle.topk_nth(raw, k, select_min, dt=dt)
     c = oracle.topk_brute(raw, k, select_min, dt=dt)
-    for x, y in ((a, b), (a, c)):
+    d = oracle.topk_nth_mt(raw, k, select_min, dt=dt)[:2]
+    for x, y in ((a, b), (a, c), (a, d)):
         assert np.array_equal(x[0], y[0]) and np.array_equal(x[1], y[1])
+
+
+def test_nth_mt_matches_sort_on_large_tied_rows():
+    """The all-cores baseline variant (chunked nth_element + merge) equals the sort oracle where
+    chunks cut through long runs of ties (a wrong chunk merge or tie rule would differ)."""
+    x = gen.adversarial_f32(5, 300_001, m_bits=26)      # 64 distinct values, ~4.7K ties each
+    for k in (1, 999, 4688, 50_000, 300_001):
+        a = oracle.topk_sort(x, k)
+        v, i, th = oracle.topk_nth_mt(x, k)
+        assert th >= 1
+        assert np.array_equal(a[0], v) and np.array_equal(a[1], i)
 
 
 # ---------------------------------------------------------------------------------------------
