@@ -501,6 +501,8 @@ def launch_names(plan):
         return ["trivial_copy"], [True]
     if plan["engine"] == 4:
         return ["gridselect_kernel (GridSelect, P:188-204)"], [True]
+    if plan["engine"] == 5:
+        return ["batch_kernel (sample + window stream + finish)", "cluster_kernel (fallback rows)"], [True, False]
     P = plan["passes"]
     L = plan["launches"]
     if L not in (P + 1, P + 3):  # window pass + tail_q grid passes + one cluster-engine tail launch

@@ -120,6 +120,34 @@ Plan make_plan(const SelectArgs& a) {
   }
   p.off_samp = p.off_bidx + align_up((size_t)2 * a.batch * p.cap_alloc * isz, 256);
   p.bytes = p.off_samp + align_up((size_t)a.batch * p.nsamp * (key_bytes(a.kind) == 8 ? 8 : 4), 256);
+  // batched engine (engine_batch.cuh): qualifies by shape when the window of every row is expected
+  // to fit the per-row finish capacity; the fallback for missed rows uses the regions above
+  p.batch_ok = 0;
+  p.off_bcnt = p.off_bslot = p.off_bsidx = p.bytes;
+  if (!a.in_idx && a.window >= 0 && (a.engine == 0 || a.engine == 5) && a.len >= (int64_t(1) << 14) &&
+      a.len < (int64_t(1) << 31)) {
+    const int es = key_bytes(a.kind), vec = 16 / es;
+    int64_t ns = std::min<int64_t>(std::max<int64_t>(a.len / 128, 4096), 16384);
+    ns = std::min<int64_t>(ns, a.len / 2) / 32 * 32;
+    if (es == 8) ns = std::min<int64_t>(ns, 8192);
+    const double f = (double)a.k / (double)a.len, r = f * (double)ns;
+    const double rhi = std::ceil(r + 4.0 * std::sqrt(r * (1.0 - f)) + 8.0);
+    const double per_row = rhi / (double)ns * (double)a.len;  // expected entries <= hi
+    if (ns >= 1024 && rhi < (double)(ns - 1) && per_row <= 0.5 * batch_fcap_host(a.kind)) {
+      const int64_t chunk = (int64_t)kBatchBlock * kBatchUnroll * vec;
+      const double e_slot = (double)kBatchUnroll * 32 * vec * rhi / (double)ns;
+      p.batch_ok = 1;
+      p.bnsamp = (int)ns;
+      p.cpc = (int)((a.len + chunk - 1) / chunk);
+      p.nwc = p.cpc * kBatchWarps;
+      p.scap = (int)align_up((size_t)std::ceil(e_slot + 6.0 * std::sqrt(e_slot) + 8.0), 4);
+      const size_t nslot = (size_t)a.batch * p.nwc;
+      p.off_bcnt = p.bytes;
+      p.off_bslot = p.off_bcnt + align_up(nslot * 2, 256);
+      p.off_bsidx = p.off_bslot + align_up(nslot * p.scap * es, 256);
+      p.bytes = p.off_bsidx + align_up(nslot * p.scap * 4, 256);
+    }
+  }
   return p;
 }
 
@@ -142,9 +170,21 @@ static int auto_cluster_size(const SelectArgs& a) {
 
 constexpr double kTailPerCTA = 4096.0;  // expected window entries per cluster-tail CTA
 
+static bool batch_aligned(const SelectArgs& a) {
+  return ((uintptr_t)a.keys % 16) == 0 && ((size_t)a.len * key_bytes(a.kind)) % 16 == 0;
+}
+
 static void choose_launch(const SelectArgs& a, Plan& p) {
   if (p.engine == 3 || p.engine == 4) return;
-  p.engine = a.engine > 0 ? a.engine : auto_engine(a);
+  // batched engine: explicit, or AUTO for batches with enough 64 KiB chunks to cover the SMs
+  if (p.batch_ok && batch_aligned(a) && (a.trace == nullptr || a.engine == 5) &&
+      (a.engine == 5 || (a.engine == 0 && a.batch >= 2 && (int64_t)a.batch * p.cpc >= num_sms()))) {
+    p.engine = 5;
+    p.csize = auto_cluster_size(a);  // fallback launch (cluster engine)
+    p.nsamp = p.bnsamp;
+    return;
+  }
+  p.engine = a.engine > 0 && a.engine != 5 ? a.engine : auto_engine(a);
   if (p.engine == 2) {
     p.csize = auto_cluster_size(a);
     return;
@@ -200,7 +240,7 @@ static airtopk_status validate(const SelectArgs& a) {
   if (!a.keys || !a.out_vals || !a.out_idx) return AIRTOPK_EINVAL;
   if (a.batch < 1 || a.len < 1 || a.k < 1 || a.k > a.len) return AIRTOPK_EINVAL;
   if (a.alpha < 0) return AIRTOPK_EINVAL;
-  if (a.engine < 0 || a.engine > 4 || a.engine == 3) return AIRTOPK_EINVAL;
+  if (a.engine < 0 || a.engine > 5 || a.engine == 3) return AIRTOPK_EINVAL;
   if (a.engine == 4 && !gridselect_supported(a)) return AIRTOPK_EINVAL;
   if (a.window < -1 || a.window > 1) return AIRTOPK_EINVAL;
   if (a.early_stop < -1 || a.early_stop > 0) return AIRTOPK_EINVAL;
@@ -237,7 +277,9 @@ static airtopk_status run(const SelectArgs& a, void* ws, size_t ws_bytes, cudaSt
   }
   choose_launch(a, p);
   if (p.engine == 2 && (p.csize < 1 || p.csize > 16 || (p.csize & (p.csize - 1)))) return AIRTOPK_EINVAL;
-  cudaError_t e = (p.engine == 2) ? run_cluster(a, p, ws, s) : run_grid(a, p, ws, s);
+  if (a.engine == 5 && p.engine != 5) return AIRTOPK_EINVAL;  // batched engine requested, shape not eligible
+  cudaError_t e = (p.engine == 2) ? run_cluster(a, p, ws, s) : (p.engine == 5) ? run_batch(a, p, ws, s)
+                                                                               : run_grid(a, p, ws, s);
   if (e == cudaSuccess && a.status) e = collect_status(a, p, ws, s);
   return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
 }
@@ -462,7 +504,7 @@ airtopk_status airtopk_describe(airtopk_dtype dtype, int64_t batch, int64_t len,
                                 const airtopk_options* opt, airtopk_plan* out) {
   if (!out) return AIRTOPK_EINVAL;
   int64_t dummy = 0;
-  SelectArgs a = make_args((const void*)1, (int)dtype, batch, len, k, 1, (void*)1, &dummy, opt);
+  SelectArgs a = make_args((const void*)256, (int)dtype, batch, len, k, 1, (void*)1, &dummy, opt);
   airtopk_status st = validate(a);
   if (st != AIRTOPK_OK) return st;
   Plan p = make_plan(a);
@@ -471,9 +513,10 @@ airtopk_status airtopk_describe(airtopk_dtype dtype, int64_t batch, int64_t len,
   std::memset(out, 0, sizeof(*out));
   out->engine = p.engine;
   out->passes = p.P;
-  out->launches = (p.engine == 3 || p.engine == 4) ? 1 : (p.engine == 2 ? 1 : (p.tail ? 3 + p.tail_q : p.P + 1 + (p.nsamp > 0 ? 2 : 0)));
+  out->launches = (p.engine == 3 || p.engine == 4) ? 1 : (p.engine == 2 ? 1 : p.engine == 5 ? 2
+                  : (p.tail ? 3 + p.tail_q : p.P + 1 + (p.nsamp > 0 ? 2 : 0)));
   out->ctas_per_row = (p.engine == 1 || p.engine == 4) ? p.cpr : 0;
-  out->cluster_size = (p.engine == 2 || p.tail) ? p.csize : 0;
+  out->cluster_size = (p.engine == 2 || p.engine == 5 || p.tail) ? p.csize : 0;
   out->index_bits = p.IB;
   out->buffer_cap = p.cap_rule;
   out->workspace_bytes = bytes;

@@ -47,7 +47,13 @@ struct Plan {
   int tail;          // grid engine: finish after the window pass with one cluster-engine launch
   int tail_q;        // ... after the grid passes q < tail_q (0: right after the window pass)
   int tma;           // grid engine: stream rows through bulk-copy (TMA) shared rings, 1 CTA/SM
-  size_t off_state, off_hist, off_bcode, off_bidx, off_samp, bytes;
+  // batched engine (engine 5, engine_batch.cuh): eligible by shape; slot geometry
+  int batch_ok;      // the shape qualifies (alignment is checked at run time)
+  int bnsamp;        // samples per row
+  int cpc;           // 64 KiB chunks per row
+  int nwc;           // (chunk, warp) slots per row
+  int scap;          // entries per slot
+  size_t off_state, off_hist, off_bcode, off_bidx, off_samp, off_bcnt, off_bslot, off_bsidx, bytes;
 };
 
 // cudaFuncSetAttribute once per (kernel, current device, attribute, value): the runtime applies
@@ -64,6 +70,10 @@ int key_bytes(int kind);
 Plan make_plan(const SelectArgs& a);
 cudaError_t run_grid(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 cudaError_t run_cluster(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
+cudaError_t run_batch(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
+// batched engine constants shared with the host plan (engine_batch.cuh)
+constexpr int kBatchBlock = 1024, kBatchWarps = 32, kBatchUnroll = 4;
+inline int batch_fcap_host(int kind) { return kBatchBlock * (kind == 3 ? 8 : 16); }
 cudaError_t run_trivial(const SelectArgs& a, cudaStream_t s);
 // K entries that sort last in the selection order (multi-GPU shard shorter than K): value bits of the
 // maximum code, indices pad_base + j

@@ -46,7 +46,8 @@ struct ClusterParams {
   int nclusters;
   int early_stop;  // 0 on, -1 off (ablation)
   int64_t idx_off; // added to every output index (airtopk_select_shard)
-  int tail;      // 1: continue rows after the grid engine's window pass
+  int tail;      // 1: continue rows after the grid engine's window pass;
+                 // 2: fallback after the batched engine: only rows with win_state == 3, from L
   int tail_q;    // tail mode: the grid engine ran passes q < tail_q after the window pass
   int timing_stride;  // int64 slots per CTA in `timing` (8; 24 with the merge-phase stamps, debug)
   int64_t* timing;  // optional: per CTA [globaltimer at start, at end, rows done, passes run, end of passes 1-4]
@@ -102,11 +103,12 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
 
   for (int64_t row = cid; row < p.batch; row += p.nclusters) {
     RowState* st = p.st + row;
+    if (p.tail == 2 && st->win_state != 3) continue;  // (cluster-uniform) finished by the batched engine
     unsigned long long K = kk, C = N, Cp = N, tcode = 0, tidx = 0;
     int stop1 = 0, src1 = 0;  // src1: 0 = the input row L, s + 1 = candidate buffer slot s
     int q0 = 0;
-    const int ws = p.tail ? st->win_state : 0;
-    if (!p.tail) {  // standalone: the row's counters start at zero (no memset launch before the kernel)
+    const int ws = p.tail == 1 ? st->win_state : 0;
+    if (p.tail != 1) {  // standalone: the row's counters start at zero (no memset launch before the kernel)
       if (crank == 0 && tid == 0) {
         st->out_count = 0;
         st->buf_count[0] = 0;
@@ -115,7 +117,7 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
       }
       cl.sync();
     }
-    if (p.tail && (ws == 1 || p.tail_q > 0)) {
+    if (p.tail == 1 && (ws == 1 || p.tail_q > 0)) {
       // continue the row from its state: after the window pass (which scanned pass 1 over the window
       // buffer) or after the grid passes q < tail_q
       K = st->K;
@@ -308,7 +310,9 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   p.early_stop = a.early_stop;
   p.idx_off = a.idx_off;
   p.tail_q = pl.tail_q;
-  p.timing = a.trace;  // cluster engine: the trace buffer receives per-CTA timing instead
+  // standalone cluster engine: the trace buffer receives per-CTA timing instead (not in tail /
+  // fallback mode: the trace then belongs to the engine that ran before)
+  p.timing = tail ? nullptr : a.trace;
   p.timing_stride = getenv("AIRTOPK_CLUSTER_TIMING") ? 24 : 8;
 
   cudaLaunchConfig_t cfg = {};

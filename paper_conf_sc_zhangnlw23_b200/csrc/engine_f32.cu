@@ -1,10 +1,12 @@
 // Grid- and cluster-engine kernels instantiated for key type F32 (see engine_grid.cuh).
+#include "engine_batch.cuh"
 #include "engine_cluster.cuh"
 #include "engine_grid.cuh"
 
 namespace airtopk {
 AIRTOPK_INSTANTIATE_GRID(K_F32)
 AIRTOPK_INSTANTIATE_CLUSTER(K_F32)
+AIRTOPK_INSTANTIATE_BATCH(K_F32)
 
 int grid_occupancy_f32(int idx64) {
   int n = 0;

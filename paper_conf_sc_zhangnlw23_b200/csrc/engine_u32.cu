@@ -1,8 +1,10 @@
 // Grid- and cluster-engine kernels instantiated for key type U32 (see engine_grid.cuh).
+#include "engine_batch.cuh"
 #include "engine_cluster.cuh"
 #include "engine_grid.cuh"
 
 namespace airtopk {
 AIRTOPK_INSTANTIATE_GRID(K_U32)
 AIRTOPK_INSTANTIATE_CLUSTER(K_U32)
+AIRTOPK_INSTANTIATE_BATCH(K_U32)
 }  // namespace airtopk
