@@ -5,6 +5,7 @@
 // stream (the iteration-fused property: the CPU only launches kernels, P:50/P:142/P:158).
 #include <algorithm>
 #include <cstdlib>
+#include <map>
 #include <mutex>
 #include <set>
 #include <tuple>
@@ -50,6 +51,28 @@ cudaError_t func_attr(const void* f, cudaFuncAttribute attr, int value) {
     done.insert(key);
   }
   return e;
+}
+
+namespace {
+std::mutex g_occ_mu;
+std::map<std::tuple<const void*, int, int>, int> g_occ;
+}  // namespace
+
+bool occ_cache_get(const void* f, int param, int* out) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return false;
+  std::lock_guard<std::mutex> g(g_occ_mu);
+  auto it = g_occ.find(std::make_tuple(f, dev, param));
+  if (it == g_occ.end()) return false;
+  *out = it->second;
+  return true;
+}
+
+void occ_cache_put(const void* f, int param, int value) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return;
+  std::lock_guard<std::mutex> g(g_occ_mu);
+  g_occ[std::make_tuple(f, dev, param)] = value;
 }
 
 int num_sms() {
@@ -123,7 +146,7 @@ Plan make_plan(const SelectArgs& a) {
   // batched engine (engine_batch.cuh): qualifies by shape when the window of every row is expected
   // to fit the per-row finish capacity; the fallback for missed rows uses the regions above
   p.batch_ok = 0;
-  p.off_bcnt = p.off_bslot = p.off_bsidx = p.bytes;
+  p.off_bcnt = p.off_bslot = p.off_bsidx = p.off_bfail = p.bytes;
   if (!a.in_idx && a.window >= 0 && (a.engine == 0 || a.engine == 5) && a.len >= (int64_t(1) << 14) &&
       a.len < (int64_t(1) << 31)) {
     const int es = key_bytes(a.kind), vec = 16 / es;
@@ -133,19 +156,21 @@ Plan make_plan(const SelectArgs& a) {
     const double f = (double)a.k / (double)a.len, r = f * (double)ns;
     const double rhi = std::ceil(r + 4.0 * std::sqrt(r * (1.0 - f)) + 8.0);
     const double per_row = rhi / (double)ns * (double)a.len;  // expected entries <= hi
-    if (ns >= 1024 && rhi < (double)(ns - 1) && per_row <= 0.5 * batch_fcap_host(a.kind)) {
-      const int64_t chunk = (int64_t)kBatchBlock * kBatchUnroll * vec;
-      const double e_slot = (double)kBatchUnroll * 32 * vec * rhi / (double)ns;
+    if (ns >= 1024 && rhi < (double)(ns - 1) && per_row <= 0.5 * kBatchFcap) {
+      const int64_t chunk = kBatchStage / es;
+      const double e_slot = (double)(kBatchStage / 16) * vec / kBatchSlotWarps * rhi / (double)ns;
       p.batch_ok = 1;
       p.bnsamp = (int)ns;
       p.cpc = (int)((a.len + chunk - 1) / chunk);
-      p.nwc = p.cpc * kBatchWarps;
-      p.scap = (int)align_up((size_t)std::ceil(e_slot + 6.0 * std::sqrt(e_slot) + 8.0), 4);
+      p.nwc = p.cpc * kBatchSlotWarps;
+      // multiple of 16 entries: slots start on 32-byte sectors (the writers pad to whole sectors)
+      p.scap = (int)align_up((size_t)std::ceil(e_slot + 6.0 * std::sqrt(e_slot) + 8.0), 16);
       const size_t nslot = (size_t)a.batch * p.nwc;
       p.off_bcnt = p.bytes;
       p.off_bslot = p.off_bcnt + align_up(nslot * 2, 256);
       p.off_bsidx = p.off_bslot + align_up(nslot * p.scap * es, 256);
-      p.bytes = p.off_bsidx + align_up(nslot * p.scap * 4, 256);
+      p.off_bfail = p.off_bsidx + align_up(nslot * p.scap * 4, 256);
+      p.bytes = p.off_bfail + align_up((size_t)(a.batch + 1) * 4, 256);
     }
   }
   return p;
@@ -178,7 +203,7 @@ static void choose_launch(const SelectArgs& a, Plan& p) {
   if (p.engine == 3 || p.engine == 4) return;
   // batched engine: explicit, or AUTO for batches with enough 64 KiB chunks to cover the SMs
   if (p.batch_ok && batch_aligned(a) && (a.trace == nullptr || a.engine == 5) &&
-      (a.engine == 5 || (a.engine == 0 && a.batch >= 2 && (int64_t)a.batch * p.cpc >= num_sms()))) {
+      (a.engine == 5 || (a.engine == 0 && a.window == 0 && a.batch >= 2 && (int64_t)a.batch * p.cpc >= num_sms()))) {
     p.engine = 5;
     p.csize = auto_cluster_size(a);  // fallback launch (cluster engine)
     p.nsamp = p.bnsamp;

@@ -50,10 +50,10 @@ struct Plan {
   // batched engine (engine 5, engine_batch.cuh): eligible by shape; slot geometry
   int batch_ok;      // the shape qualifies (alignment is checked at run time)
   int bnsamp;        // samples per row
-  int cpc;           // 64 KiB chunks per row
+  int cpc;           // 32 KiB chunks per row
   int nwc;           // (chunk, warp) slots per row
   int scap;          // entries per slot
-  size_t off_state, off_hist, off_bcode, off_bidx, off_samp, off_bcnt, off_bslot, off_bsidx, bytes;
+  size_t off_state, off_hist, off_bcode, off_bidx, off_samp, off_bcnt, off_bslot, off_bsidx, off_bfail, bytes;
 };
 
 // cudaFuncSetAttribute once per (kernel, current device, attribute, value): the runtime applies
@@ -64,6 +64,11 @@ cudaError_t func_attr(F* func, cudaFuncAttribute attr, int value) {
   return func_attr(reinterpret_cast<const void*>(func), attr, value);
 }
 
+// Memoised occupancy queries (per kernel, current device and parameter): the runtime queries cost
+// microseconds of host time, which the small configs (c1, c2 shards) cannot afford per call.
+bool occ_cache_get(const void* f, int param, int* out);
+void occ_cache_put(const void* f, int param, int value);
+
 int key_bits(int kind);
 int num_sms();  // SMs of the current device (cached per thread)
 int key_bytes(int kind);
@@ -72,8 +77,10 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t 
 cudaError_t run_cluster(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 cudaError_t run_batch(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 // batched engine constants shared with the host plan (engine_batch.cuh)
-constexpr int kBatchBlock = 1024, kBatchWarps = 32, kBatchUnroll = 4;
-inline int batch_fcap_host(int kind) { return kBatchBlock * (kind == 3 ? 8 : 16); }
+constexpr int kBatchBlock = 1024, kBatchWarps = 32;
+constexpr int kBatchSlotWarps = 16;  // warps per consumer group = (chunk, warp) slots per chunk
+constexpr int kBatchStage = 32768;   // bytes per chunk (one bulk-copy ring stage)
+constexpr int kBatchFcap = 16384;    // entries (results + window members) one row may stage in the finish
 cudaError_t run_trivial(const SelectArgs& a, cudaStream_t s);
 // K entries that sort last in the selection order (multi-GPU shard shorter than K): value bits of the
 // maximum code, indices pad_base + j

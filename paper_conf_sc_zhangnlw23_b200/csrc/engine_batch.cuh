@@ -9,11 +9,13 @@
 //
 //   A  sample: CTA r (rows r, r + G, ...) draws S stratified runs of 32 keys of its row, selects the
 //      sample order statistics around the expected rank of the K-th key and stores the window
-//      [lo, hi] (the same estimator and 4-sigma+8 margin as sample_kernel); CTAs first issue L2 bulk
-//      prefetches of the chunks they stream first, so HBM works during the sampling latency.
-//   B  stream: the batch is cut into 64 KiB chunks, chunk c -> CTA c mod G (grid-stride over the
+//      [lo, hi] (the same estimator and 4-sigma+8 margin as sample_kernel) by MSD digit histograms
+//      of the samples and a counting rank once <= 1024 candidates remain.
+//   B  stream: the batch is cut into 32 KiB chunks, chunk c -> CTA c mod G (grid-stride over the
 //      flattened batch: no wave quantisation, every SM streams ~equal bytes; the CTAs stream one
-//      compact advancing region of HBM). Per element ONE compare of the raw key bits against the
+//      compact advancing region of HBM). Each CTA pulls its chunks through a ring of 6 bulk-copy
+//      stages (cp.async.bulk, TMA engine, mbarrier full/empty handshake: 192 KiB in flight per SM,
+//      the first 4 issued before phase A). Per element ONE compare of the raw key bits against the
 //      transformed threshold hi (exact); the rare flagged keys (code <= hi) are written by their
 //      warp to a FIXED slot of its (chunk, warp) — no atomics, no queues, no block barriers in the
 //      streaming loop — and the warp stores the slot's count.
@@ -24,6 +26,10 @@
 //      register-resident entries: per pass a 2048-bin shared histogram, the inclusive scan and the
 //      target digit j with psum[j-1] < K <= psum[j] (Alg1 L24-28), filter (digit < j ->
 //      result, == j -> candidate), early stop when K == C.
+//
+// Code size matters here: phases A and C run once per row on a cold instruction cache (measured:
+// fully unrolled register-array versions spent ~10 us per phase fetching straight-line code), so
+// their loops stay rolled and their data lives in shared memory.
 //
 // Exactness never depends on the sample: a row whose window misses (or overflows a slot or the
 // finish capacity, or had no usable window) is marked win_state = 3 and the next, already enqueued,
@@ -41,17 +47,27 @@ namespace airtopk {
 
 constexpr int kBBlock = kBatchBlock;          // threads per CTA (1 CTA per SM)
 constexpr int kBWarps = kBBlock / 32;
-constexpr int kBUnroll = kBatchUnroll;        // 16-byte vectors per thread per chunk (64 KiB chunks)
 static_assert(kBWarps == kBatchWarps, "host/device slot geometry");
-constexpr int kBChunkVec = kBBlock * kBUnroll;  // 16-byte vectors per chunk
-constexpr int kBWarpElems32 = 32 * kBUnroll * 4;  // f32 elements per (chunk, warp) slot: 512
-
-// entries (results + window members) one row may stage in the finish: PER per thread in registers
-template <int KIND>
-__host__ __device__ constexpr int batch_per_thread() { return sizeof(typename KT<KIND>::U) == 8 ? 8 : 16; }
-template <int KIND>
-__host__ __device__ constexpr int batch_fcap() { return kBBlock * batch_per_thread<KIND>(); }
-static_assert(batch_fcap<K_F64>() == kBatchBlock * 8 && batch_fcap<K_F32>() == kBatchBlock * 16, "batch_fcap_host");
+constexpr unsigned kBStage = kBatchStage;     // bytes per bulk-copy ring stage = one chunk of a row
+constexpr int kBStages = 6;                   // ring depth: 192 KiB in flight per SM
+constexpr int kBPre = 4;                      // stages issued before the sampling phase
+#ifndef AIRTOPK_BATCH_L2PRE
+#define AIRTOPK_BATCH_L2PRE 0  // measured: L2 prefetches during phase A slow the sampling, stream unchanged
+#endif
+constexpr int kBL2Pre = AIRTOPK_BATCH_L2PRE;  // further chunks per CTA prefetched into L2 during phase A
+// Phase B consumers: two groups of 16 warps take alternate stages, 4 vectors per thread each (a
+// warp's per-stage overhead — barrier wait, count store, loop — is amortised over 2 KiB).
+constexpr int kBGroups = 2;
+constexpr int kBGWarps = kBWarps / kBGroups;
+constexpr int kBGThreads = kBGWarps * 32;
+constexpr int kBVT = (int)(kBStage / 16 / kBGThreads);  // 16-byte vectors per thread per stage
+static_assert(kBVT * 16 * kBGThreads == (int)kBStage, "stage = group threads x kBVT vectors");
+static_assert(kBStages % kBGroups == 0, "a stage always belongs to the same group");
+static_assert(kBGWarps == kBatchSlotWarps, "host/device slot geometry");
+constexpr int kBFcap = kBatchFcap;            // entries (results + members) one row may stage in the finish
+constexpr int kBBrute = 1024;                 // sample-rank selection: brute-force rank below this many
+constexpr size_t kBRingBytes = (size_t)kBStages * kBStage;
+static_assert((size_t)kMaxSamples * 4 <= (size_t)(kBStages - kBPre) * kBStage, "samples fit the unused stages");
 
 struct BatchParams {
   const void* keys;
@@ -62,128 +78,223 @@ struct BatchParams {
   int64_t* out_idx;
   int64_t idx_off;
   RowState* st;
-  unsigned short* cnt;    // [batch][nwc] entries written per (chunk, warp) slot (cap + 1 = overflow)
+  unsigned short* cnt;    // [batch][nwc] entries written per (chunk, group warp) slot (cap + 1 = overflow)
   void* scode;            // [batch][nwc][scap] codes
   unsigned* sidx;         // [batch][nwc][scap] row indices
-  int nwc;                // slots per row = chunks per row * kBWarps
+  int nwc;                // slots per row = chunks per row * kBGWarps
   int scap;               // entries per slot
   int cpc;                // chunks per row
   int nsamp;              // samples per row
   int early_stop;         // 0 on, -1 off
+  unsigned* fail;         // [0] = number of rows for the fallback launch, [1 + i] = those rows
   int64_t* timing;        // optional (trace buffer): per CTA globaltimer stamps of the phases
   int64_t timing_n;       // int64 entries of `timing`
 };
 
-__device__ __forceinline__ void prefetch_l2(const void* p, unsigned bytes) {
-  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+// debug timing (trace buffer): per CTA 32 %globaltimer stamps (tools/batch_timing.py)
+__device__ __forceinline__ void bstamp(const BatchParams& p, int f) {
+  if (p.timing && threadIdx.x == 0 && (int64_t)blockIdx.x * 32 + f < p.timing_n) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    p.timing[(int64_t)blockIdx.x * 32 + f] = (int64_t)t;
+  }
 }
 
-// Phase A for one row (all threads of the CTA): window [lo, hi] from the sample order statistics.
+// Shared scratch of the sampling and finish phases (static; the big arrays live in the ring).
+template <typename W>
+struct BatchShared {
+  unsigned hist[kMaxBins];
+  W brute[kBBrute];             // compacted candidates of the rank selection
+  unsigned long long tmp[kBWarps];
+  ScanResult res;
+  W wmin[kBWarps], wmax[kBWarps];
+  W result;
+  unsigned long long tot;
+  unsigned cnt, out;
+  int bad;
+};
+
+// ---------------------------------------------------------------------------------- phase A
+// Sample order statistic of rank `rank` among the samples s[0..ns) (shared memory), all threads.
+// MSD digits of up to 11 bits below the bits on which every sample agrees (prefix); once at most
+// kBBrute samples share the prefix they are compacted and ranked by counting.
+template <typename W, typename Stamp = NoStamp>
+__device__ W sample_rank(const W* s, int ns, int rank, W smin, W smax, BatchShared<W>& sh, Stamp stamp = Stamp()) {
+  constexpr int WB = 8 * (int)sizeof(W);
+  const W diff = smin ^ smax;
+  int hb = diff ? (WB - (sizeof(W) == 8 ? __clzll((long long)diff) : __clz((int)diff))) : 0;
+  W mask = (hb >= WB) ? (W)0 : (W)(~(W)0 << hb);
+  W prefix = smin & mask;
+  int cnt = ns;
+  while (true) {
+    if (hb == 0) return prefix;
+    if (cnt <= kBBrute) {
+      if (threadIdx.x == 0) sh.cnt = 0;
+      __syncthreads();
+#pragma unroll 1
+      for (int i = threadIdx.x; i < ns; i += kBBlock) {
+        const W x = s[i];
+        const bool m = (x & mask) == prefix;
+        const unsigned b = __ballot_sync(kFull, m);
+        unsigned base = 0;
+        if ((threadIdx.x & 31) == 0 && b) base = atomicAdd(&sh.cnt, (unsigned)__popc(b));
+        base = __shfl_sync(kFull, base, 0);
+        if (m) sh.brute[base + __popc(b & lanemask_lt())] = x;
+      }
+      __syncthreads();
+      stamp(3);
+      if ((int)threadIdx.x < cnt) {
+        const W x = sh.brute[threadIdx.x];
+        int less = 0, eq = 0;
+#pragma unroll 4
+        for (int j = 0; j < cnt; ++j) {
+          const W y = sh.brute[j];
+          less += y < x;
+          eq += y == x;
+        }
+        if (less <= rank && rank < less + eq) sh.result = x;
+      }
+      __syncthreads();
+      stamp(4);
+      const W r = sh.result;
+      __syncthreads();
+      return r;
+    }
+    const int shf = hb > kDigitBits ? hb - kDigitBits : 0, w = hb - shf;
+    const unsigned dm = (1u << w) - 1u;
+    for (int i = threadIdx.x; i < (1 << w); i += kBBlock) sh.hist[i] = 0;
+    __syncthreads();
+    stamp(0);
+#pragma unroll 1
+    for (int i = threadIdx.x; i < ns; i += kBBlock) {
+      const W x = s[i];
+      if ((x & mask) == prefix) atomicAdd(&sh.hist[(unsigned)(x >> shf) & dm], 1u);
+    }
+    __syncthreads();
+    stamp(1);
+    const ScanResult r = scan_choose<kBBlock>([&](int b) { return (unsigned long long)sh.hist[b]; }, 1 << w,
+                                             (unsigned long long)rank + 1, sh.tmp, &sh.res);
+    stamp(2);
+    rank -= (int)r.before;
+    cnt = (int)r.cnt;
+    prefix |= (W)r.j << shf;
+    mask |= (W)dm << shf;
+    hb = shf;
+  }
+}
+
+// Phase A for one row (all threads): window [lo, hi] from the sample order statistics.
+template <typename U>
+__device__ __forceinline__ void batch_issue(const BatchParams& p, int64_t ch, unsigned ring, int stage);
+template <typename U>
+__device__ __forceinline__ void batch_prefetch_l2(const BatchParams& p, int64_t ch);
+
 template <int KIND>
-__device__ void batch_sample_row(const BatchParams& p, int64_t row, void* scratch_v) {
+__device__ void batch_sample_row(const BatchParams& p, int64_t row, void* samp_v,
+                                 BatchShared<std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long,
+                                                                unsigned>>& sh,
+                                 int64_t issue_mine, unsigned ring) {
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
-  constexpr int PER = kMaxSamples / kBBlock;
-  __shared__ unsigned hist[2048 * kSampleHistCopies];
-  __shared__ unsigned wsum[32];
-  __shared__ W shw[8];
-  __shared__ int sh_cnt[4];
-  __shared__ W sh_red[64];
-  W* scratch = (W*)scratch_v;
+  W* s = (W*)samp_v;
   RowState* st = p.st + row;
-  const int nsamp = p.nsamp;
+  const int ns = p.nsamp;
   const U* rowp = (const U*)p.keys + row * p.len;
   const U xmask = p.sel_min ? (U)0 : (U)~(U)0;
-  constexpr int kRun = 32;
-  const int nruns = nsamp / kRun;
-  const int64_t stride = p.len / nruns;
-  W v[PER];
+  constexpr int kRun = 32;  // samples come in runs of 32 consecutive keys (one 128-byte line for f32)
+  const int64_t stride = p.len / (ns / kRun);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  W lmin = ~(W)0, lmax = 0;
+  // all of a thread's sample loads are issued before any is stored: `s` is a generic pointer the
+  // compiler cannot prove disjoint from the row, so interleaved store / load pairs would serialise
+  // one DRAM latency per sample (measured)
+  constexpr int kSPT = kMaxSamples / kBBlock;  // samples per thread (<= 16)
   {
-    U x[PER];
+    U x[kSPT];
 #pragma unroll
-    for (int t = 0; t < PER; ++t) {
-      const int slot = t * kBBlock + threadIdx.x;
-      const int run = slot / kRun, e = slot % kRun;
-      const int64_t pos = (int64_t)run * stride + (stride - kRun) / 2 + e;
-      if (run < nruns) x[t] = __ldg(rowp + pos);
+    for (int t = 0; t < kSPT; ++t) {
+      const int i = threadIdx.x + t * kBBlock;
+      x[t] = (i < ns) ? __ldg(rowp + (int64_t)(i / kRun) * stride + (stride - kRun) / 2 + (i % kRun)) : (U)0;
     }
 #pragma unroll
-    for (int t = 0; t < PER; ++t) {
-      const int slot = t * kBBlock + threadIdx.x;
-      v[t] = (slot < nsamp) ? (W)to_code_x<KIND>(x[t], xmask) : (W)0;
+    for (int t = 0; t < kSPT; ++t) {
+      const int i = threadIdx.x + t * kBBlock;
+      if (i < ns) {
+        const W c = (W)to_code_x<KIND>(x[t], xmask);
+        s[i] = c;
+        lmin = c < lmin ? c : lmin;
+        lmax = c > lmax ? c : lmax;
+      }
     }
   }
-  const int tv = (nsamp - (int)threadIdx.x + kBBlock - 1) / kBBlock;  // valid v[t]: t < tv
-  W lmin = ~(W)0, lmax = 0;
-#pragma unroll
-  for (int t = 0; t < PER; ++t) {
-    if (t < tv) {
-      lmin = v[t] < lmin ? v[t] : lmin;
-      lmax = v[t] > lmax ? v[t] : lmax;
-    }
+  bstamp(p, 1);
+  if (threadIdx.x == 0) {  // (the loads above have returned: their values are in lmin / lmax)
+    for (int i = 0; i < kBPre && i < issue_mine; ++i) batch_issue<U>(p, blockIdx.x + (int64_t)i * gridDim.x, ring, i);
+    for (int i = kBPre; i < kBPre + kBL2Pre && i < issue_mine; ++i)
+      batch_prefetch_l2<U>(p, blockIdx.x + (int64_t)i * gridDim.x);
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
-    const W a = shfl(lmin, (threadIdx.x + o) & 31), b = shfl(lmax, (threadIdx.x + o) & 31);
+    const W a = shfl(lmin, lane ^ o), b = shfl(lmax, lane ^ o);
     lmin = a < lmin ? a : lmin;
     lmax = b > lmax ? b : lmax;
   }
-  if ((threadIdx.x & 31) == 0) {
-    sh_red[threadIdx.x >> 5] = lmin;
-    sh_red[32 + (threadIdx.x >> 5)] = lmax;
+  if (lane == 0) {
+    sh.wmin[warp] = lmin;
+    sh.wmax[warp] = lmax;
   }
-  if (threadIdx.x == 0) sh_cnt[2] = 0;
   __syncthreads();
-  W smin = sh_red[0], smax = sh_red[32];
-#pragma unroll 8
-  for (int i = 1; i < kBWarps; ++i) {
-    smin = sh_red[i] < smin ? sh_red[i] : smin;
-    smax = sh_red[32 + i] > smax ? sh_red[32 + i] : smax;
+  W smin = sh.wmin[lane], smax = sh.wmax[lane];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const W a = shfl(smin, lane ^ o), b = shfl(smax, lane ^ o);
+    smin = a < smin ? a : smin;
+    smax = b > smax ? b : smax;
   }
-  // expected sample rank of the K-th key, 4-sigma (+8) binomial margin (as sample_kernel)
+  // expected sample rank of the K-th key and a 4-sigma (+8) binomial margin (as sample_kernel):
+  // a miss only costs the fallback, never exactness
   const double f = (double)p.k / (double)p.len;
-  const double r = f * nsamp;
+  const double r = f * ns;
   const double m = 4.0 * sqrt(r * (1.0 - f)) + 8.0;
   const int rlo = (int)floor(r - m), rhi = (int)ceil(r + m);
   int state = 1;
   W lo = 0, hi = 0;
-  if (rhi >= nsamp - 1) {
+  if (rhi >= ns - 1) {
     state = 3;
   } else {
-    const W diff = smin ^ smax;
-    const int hb = diff ? (8 * (int)sizeof(W) - (sizeof(W) == 8 ? __clzll((long long)diff) : __clz((int)diff))) : 0;
-    block_select_two<W, PER>(v, tv, scratch, rlo <= 0 ? -1 : rlo, rhi, smin, hb, hist, wsum, shw, sh_cnt, lo, hi);
-    if (rlo <= 0) lo = 0;
+    hi = sample_rank<W>(s, ns, rhi, smin, smax, sh, [&](int f) { bstamp(p, 16 + f); });
+    lo = rlo > 0 ? sample_rank<W>(s, ns, rlo, smin, smax, sh) : (W)0;  // none below the window if rlo <= 0
+    bstamp(p, 2);
     // estimated entries (results + members: every code <= hi) vs the finish capacity
     unsigned le = 0;
-#pragma unroll
-    for (int t = 0; t < PER; ++t) le += (t < tv) && v[t] <= hi;
+#pragma unroll 4
+    for (int i = threadIdx.x; i < ns; i += kBBlock) le += s[i] <= hi;
     le = __reduce_add_sync(kFull, le);
-    if ((threadIdx.x & 31) == 0 && le) atomicAdd(&sh_cnt[2], (int)le);
+    if (threadIdx.x == 0) sh.cnt = 0;
     __syncthreads();
-    const double est = (double)sh_cnt[2] / nsamp * (double)p.len;
-    if (est > 0.6 * (double)batch_fcap<KIND>()) state = 3;
+    if (lane == 0 && le) atomicAdd(&sh.cnt, le);
+    __syncthreads();
+    if ((double)sh.cnt / ns * (double)p.len > 0.6 * (double)kBFcap) state = 3;
   }
   if (threadIdx.x == 0) {
     st->win_lo = lo;
     st->win_hi = hi;
     st->win_state = state;
     st->out_count = 0;
-    st->buf_count[0] = 0;
-    st->buf_count[1] = 0;
     st->error = 0;
   }
   __syncthreads();
 }
 
+// ---------------------------------------------------------------------------------- phase B
 // Threshold of the raw-bit test: code(b) <= hi  <=>  (b ^ wx) <= hi (see run_pass, DF == 3).
 template <int KIND>
-__device__ __forceinline__ typename std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long, unsigned>
+__device__ __forceinline__ std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long, unsigned>
 raw_xor_for(unsigned long long hi, bool sel_min) {
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
   constexpr W S = (W)((W)1 << (KT<KIND>::R - 1));
-  constexpr W ones = (W)(U)~(U)0;
+  constexpr W ones = (W)(U)~(U)0;  // (U) again: ~ promotes 16-bit keys to int
   const W whi = (W)hi;
   if constexpr (KT<KIND>::IEEE) {
     if (sel_min) return (whi >= S) ? S : ones;
@@ -193,51 +304,71 @@ raw_xor_for(unsigned long long hi, bool sel_min) {
   }
 }
 
-// Phase B for one chunk (all threads): flag code <= hi, write the warp's flagged keys to its slot.
-template <int KIND>
-__device__ __forceinline__ void batch_stream_chunk(const BatchParams& p, int64_t row, int ci, unsigned long long hi) {
+// Chunk ch of the flattened batch into ring stage `stage` (thread 0).
+// L2 prefetch of chunk ch (no shared memory involved): phase A lasts several microseconds during
+// which HBM would idle; the chunks a CTA streams right after the ring's first stages are pulled
+// into L2 meanwhile.
+template <typename U>
+__device__ __forceinline__ void batch_prefetch_l2(const BatchParams& p, int64_t ch) {
+  const int64_t row = ch / p.cpc, ci = ch - row * p.cpc;
+  const int64_t rb = p.len * (int64_t)sizeof(U);
+  const unsigned bytes = (unsigned)min((int64_t)kBStage, rb - ci * (int64_t)kBStage);
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"((const char*)p.keys + row * rb + ci * (int64_t)kBStage),
+               "r"(bytes)
+               : "memory");
+}
+
+// The input is read exactly once: its L2 lines are marked evict-first so the (chunk, warp) slots
+// written meanwhile stay in L2 for the finish.
+template <typename U>
+__device__ __forceinline__ void batch_issue(const BatchParams& p, int64_t ch, unsigned ring, int stage) {
+  const int64_t row = ch / p.cpc, ci = ch - row * p.cpc;
+  const int64_t rb = p.len * (int64_t)sizeof(U);
+  const unsigned bytes = (unsigned)min((int64_t)kBStage, rb - ci * (int64_t)kBStage);
+  const unsigned fullb = ring + (unsigned)kBRingBytes + 8u * stage;
+  mbar_arrive_expect_tx(fullb, bytes);
+  bulk_g2s_hint(ring + stage * kBStage, (const char*)p.keys + row * rb + ci * (int64_t)kBStage, bytes, fullb,
+                l2_policy_evict_first());
+}
+
+// Flag code <= hi among this thread's vectors of a stage (gt = thread index in its group, gw =
+// warp in its group), write the warp's flagged keys to its slot. Fast path per element: one xor and
+// one min of the raw bits; the flags are only built when the minimum hits (a few lanes per stage).
+template <int KIND, bool FULL>
+__device__ __forceinline__ void batch_classify(const BatchParams& p, int64_t row, int ci, unsigned long long hi,
+                                               unsigned sbase, int nv, int gt, int gw) {
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
   constexpr int VEC = 16 / sizeof(U);
-  constexpr int NE = kBUnroll * VEC;  // elements per thread per chunk
-  using FlagT = std::conditional_t<(NE > 32), unsigned long long, unsigned>;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  using FlagT = std::conditional_t<(kBVT * VEC > 32), unsigned long long, unsigned>;
+  const int lane = gt & 31;
   const bool sel_min = p.sel_min != 0;
   const W whi = (W)hi;
   const W wx = raw_xor_for<KIND>(hi, sel_min);
-  const U xmask = sel_min ? (U)0 : (U)~(U)0;
-  const int64_t nvec = p.len / VEC;  // rows are whole 16-byte vectors (checked on the host)
-  const uint4* vp = (const uint4*)((const U*)p.keys + row * p.len);
-  const int64_t vb = (int64_t)ci * kBChunkVec + tid;
-  uint4 r[kBUnroll];
+  uint4 r[kBVT];
 #pragma unroll
-  for (int u = 0; u < kBUnroll; ++u) {
-    const int64_t v = vb + (int64_t)u * kBBlock;
-    r[u] = (v < nvec) ? ldg_stream(vp + v) : make_uint4(0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu);
-  }
-  FlagT fl = 0;
+  for (int u = 0; u < kBVT; ++u) r[u] = lds128(sbase + (unsigned)((gt + u * kBGThreads) * 16));
   W m = ~(W)0;
 #pragma unroll
-  for (int u = 0; u < kBUnroll; ++u) {
-    const bool valid = vb + (int64_t)u * kBBlock < nvec;
+  for (int u = 0; u < kBVT; ++u) {
+    const bool valid = FULL || gt + u * kBGThreads < nv;
 #pragma unroll
     for (int e = 0; e < VEC; ++e) {
       const W t = (W)((W)vec_elem<U>(r[u], e) ^ wx);
       m = (valid && t < m) ? t : m;
     }
   }
-  if (m <= whi) {
+  const size_t slot = (size_t)row * p.nwc + (size_t)ci * kBGWarps + gw;
+  int total = 0;
+  if (__any_sync(kFull, m <= whi)) {
+    FlagT fl = 0;
 #pragma unroll
-    for (int u = 0; u < kBUnroll; ++u) {
-      const bool valid = vb + (int64_t)u * kBBlock < nvec;
+    for (int u = 0; u < kBVT; ++u) {
+      const bool valid = FULL || gt + u * kBGThreads < nv;
 #pragma unroll
       for (int e = 0; e < VEC; ++e)
         if (valid && (W)((W)vec_elem<U>(r[u], e) ^ wx) <= whi) fl |= (FlagT)1 << (u * VEC + e);
     }
-  }
-  const size_t slot = (size_t)row * p.nwc + (size_t)ci * kBWarps + warp;
-  int total = 0;
-  if (__any_sync(kFull, fl != 0)) {
     const int n = (sizeof(FlagT) == 8) ? __popcll((unsigned long long)fl) : __popc((unsigned)fl);
     int incl = n;
 #pragma unroll
@@ -249,105 +380,163 @@ __device__ __forceinline__ void batch_stream_chunk(const BatchParams& p, int64_t
     int pos = incl - n;
     U* sc = (U*)p.scode + slot * p.scap;
     unsigned* si = p.sidx + slot * p.scap;
+    const U xmask = sel_min ? (U)0 : (U)~(U)0;
+    // pad the written entries to whole 32-byte sectors: a partially written L2 sector would have to
+    // be filled from DRAM when the finish reads it (measured: ~7 us of the finish)
+    constexpr int kSec = 32 / (sizeof(U) < 4 ? sizeof(U) : 4);
+    const int padded = min(p.scap, (total + kSec - 1) / kSec * kSec);
+    const unsigned long long keep = l2_policy_evict_last();
+    for (int q = total + lane; q < padded; q += 32) {
+      st_keep(sc + q, (U)0, keep);
+      st_keep(si + q, 0u, keep);
+    }
+#pragma unroll 1
     while (fl) {
       const int b = ((sizeof(FlagT) == 8) ? __ffsll((long long)fl) : __ffs((int)fl)) - 1;
       fl &= fl - 1;
       if (pos < p.scap) {
         const int u = b / VEC, e = b % VEC;
-        uint4 vv = r[0];
-#pragma unroll
-        for (int i = 1; i < kBUnroll; ++i) vv = (u == i) ? r[i] : vv;
-        U raw = vec_elem<U>(vv, 0);
-#pragma unroll
-        for (int i = 1; i < VEC; ++i) raw = (e == i) ? vec_elem<U>(vv, i) : raw;
-        sc[pos] = to_code_x<KIND>(raw, xmask);
-        si[pos] = (unsigned)((vb + (int64_t)u * kBBlock) * VEC + e);
+        const unsigned a = sbase + (unsigned)((gt + u * kBGThreads) * 16 + e * (int)sizeof(U));
+        U raw;
+        if constexpr (sizeof(U) == 2) { unsigned short t; asm volatile("ld.shared.u16 %0, [%1];" : "=h"(t) : "r"(a)); raw = t; }
+        else if constexpr (sizeof(U) == 4) { unsigned t; asm volatile("ld.shared.u32 %0, [%1];" : "=r"(t) : "r"(a)); raw = t; }
+        else { unsigned long long t; asm volatile("ld.shared.u64 %0, [%1];" : "=l"(t) : "r"(a)); raw = t; }
+        st_keep(sc + pos, to_code_x<KIND>(raw, xmask), keep);
+        st_keep(si + pos, (unsigned)((int64_t)ci * (kBStage / sizeof(U)) + (int64_t)(gt + u * kBGThreads) * VEC + e), keep);
       }
       ++pos;
     }
   }
-  if (lane == 0) p.cnt[slot] = (unsigned short)(total > p.scap ? p.scap + 1 : total);
+  if (lane == 0) st_keep(p.cnt + slot, (unsigned short)(total > p.scap ? p.scap + 1 : total), l2_policy_evict_last());
 }
 
-// Phase C for one row (all threads): gather, check the window, emit results, select the members.
+// ---------------------------------------------------------------------------------- phase C
+// One row (all threads): gather, check the window, emit results, select the members.
 template <int KIND>
-__device__ void batch_finish_row(const BatchParams& p, int64_t row, void* stage) {
+__device__ void batch_finish_row(const BatchParams& p, int64_t row, void* stage,
+                                 BatchShared<std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long,
+                                                                unsigned>>& sh) {
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
-  constexpr int PER = batch_per_thread<KIND>();
-  constexpr int FCAP = batch_fcap<KIND>();
-  __shared__ unsigned long long s_tmp[kBWarps];
-  __shared__ ScanResult s_res;
-  __shared__ unsigned s_hist[kMaxBins];
-  __shared__ unsigned long long s_tot[2];
-  __shared__ unsigned s_out;
-  __shared__ int s_bad;
-  const int tid = threadIdx.x, lane = tid & 31;
+  constexpr int WB = 8 * (int)sizeof(W);
+  constexpr int PER = kBFcap / kBBlock;
+  static_assert(PER <= 32, "valid bits per thread");
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   RowState* st = p.st + row;
-  if (st->win_state != 1) return;  // (uniform) no window: the fallback launch selects the row
-  const unsigned long long lo = st->win_lo, hi = st->win_hi;
-  U* stc = (U*)stage;
-  unsigned* sti = (unsigned*)((char*)stage + (size_t)FCAP * sizeof(U));
-  // --- slot counts -> offsets (thread t owns slots [t*per, (t+1)*per)) ---
-  const int nwc = p.nwc;
-  const int per = (nwc + kBBlock - 1) / kBBlock;
-  const unsigned short* cnt = p.cnt + (size_t)row * nwc;
-  const int s0 = min(nwc, tid * per), s1 = min(nwc, s0 + per);
-  unsigned long long mine = 0;
-  int bad = 0;
-  for (int s = s0; s < s1; ++s) {
-    const int c = cnt[s];
-    bad |= c > p.scap;
-    mine += (unsigned)c;
-  }
-  if (tid == 0) s_bad = 0;
-  __syncthreads();
-  if (__any_sync(kFull, bad) && lane == 0) s_bad = 1;
-  unsigned long long total;
-  unsigned long long off = block_exclusive_scan<kBBlock>(mine, s_tmp, total);
-  if (s_bad || total > (unsigned long long)FCAP || total < (unsigned long long)p.k) {
-    if (tid == 0) st->win_state = 3;  // slot overflow / too many entries / window below the K-th key
+  auto fail = [&]() {  // the fallback launch selects the row from L (nothing was emitted)
+    if (tid == 0) {
+      st->win_state = 3;
+      p.fail[1 + atomicAdd(p.fail, 1u)] = (unsigned)row;
+    }
     __syncthreads();
+  };
+  if (st->win_state != 1) {  // (uniform) no usable window
+    fail();
     return;
   }
-  // --- gather the entries into shared memory (L2 reads), then into registers ---
-  for (int s = s0; s < s1; ++s) {
-    const int c = cnt[s];
-    const U* sc = (const U*)p.scode + ((size_t)row * nwc + s) * p.scap;
-    const unsigned* si = p.sidx + ((size_t)row * nwc + s) * p.scap;
-    for (int j = 0; j < c; ++j) {
-      stc[off + j] = __ldcg(sc + j);
-      sti[off + j] = __ldcg(si + j);
-    }
-    off += c;
+  const W lo = (W)st->win_lo;
+  bstamp(p, 20);
+  U* stc = (U*)stage;
+  unsigned* sti = (unsigned*)((char*)stage + (size_t)kBFcap * sizeof(U));
+  // --- gather: warp w takes slots w*32 + lane + r*kBBlock (coalesced counts, loaded for kGR
+  // rounds at once), a warp scan places its slots' entries, ONE shared atomic per warp and round
+  // reserves staging room (the order of entries is irrelevant to the selection), and every entry
+  // load of a round is in flight together ---
+  const int nwc = p.nwc;
+  const unsigned short* cnt = p.cnt + (size_t)row * nwc;
+  if (tid == 0) {
+    sh.cnt = 0;
+    sh.bad = 0;
   }
   __syncthreads();
-  const int n = (int)total;
-  U vc[PER];
-  unsigned vi[PER];
-  unsigned valid = 0;  // bit t: register slot t holds an entry
-  unsigned nres = 0;   // results (code < lo) held by this thread
+  bstamp(p, 21);
+  // per warp iteration: kGR slots per lane; offsets first (scans + one shared atomic per round),
+  // then every entry load of the iteration, then the stores — the staging pointer is generic, so
+  // interleaved stores would serialise the loads (measured: ~5 us)
+  constexpr int kGR = 2, kGJ = 4;
+#pragma unroll 1
+  for (int base = warp * 32 + lane; base - lane < nwc; base += kGR * kBBlock) {
+    int cc[kGR];
+    unsigned o[kGR];
 #pragma unroll
-  for (int t = 0; t < PER; ++t) {
-    const int e = t * kBBlock + tid;
-    vc[t] = (e < n) ? stc[e] : (U)0;
-    vi[t] = (e < n) ? sti[e] : 0u;
-    if (e < n) {
-      valid |= 1u << t;
-      nres += ((W)vc[t] < (W)lo);
+    for (int r = 0; r < kGR; ++r) {
+      const int sl = base + r * kBBlock;
+      cc[r] = sl < nwc ? (int)__ldcg(cnt + sl) : 0;
     }
+#pragma unroll
+    for (int r = 0; r < kGR; ++r) {
+      if (cc[r] > p.scap) sh.bad = 1;
+      cc[r] = min(cc[r], p.scap);
+      int incl = cc[r];
+#pragma unroll
+      for (int q = 1; q < 32; q <<= 1) {
+        const int y = __shfl_up_sync(kFull, incl, q);
+        if (lane >= q) incl += y;
+      }
+      const int tot = __shfl_sync(kFull, incl, 31);
+      unsigned b = 0;
+      if (lane == 0 && tot) b = atomicAdd(&sh.cnt, (unsigned)tot);
+      o[r] = __shfl_sync(kFull, b, 0) + (unsigned)(incl - cc[r]);
+    }
+    U vc[kGR][kGJ];
+    unsigned vi[kGR][kGJ];
+#pragma unroll
+    for (int r = 0; r < kGR; ++r) {
+      const size_t src = ((size_t)row * nwc + base + r * kBBlock) * p.scap;
+#pragma unroll
+      for (int j = 0; j < kGJ; ++j) {
+        if (j < cc[r]) {
+          vc[r][j] = __ldcg((const U*)p.scode + src + j);
+          vi[r][j] = __ldcg(p.sidx + src + j);
+        }
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < kGR; ++r) {
+#pragma unroll
+      for (int j = 0; j < kGJ; ++j) {
+        if (j < cc[r] && o[r] + j < (unsigned)kBFcap) {
+          stc[o[r] + j] = vc[r][j];
+          sti[o[r] + j] = vi[r][j];
+        }
+      }
+      const size_t src = ((size_t)row * nwc + base + r * kBBlock) * p.scap;
+#pragma unroll 1
+      for (int j = kGJ; j < cc[r]; ++j) {
+        if (o[r] + j < (unsigned)kBFcap) {
+          stc[o[r] + j] = __ldcg((const U*)p.scode + src + j);
+          sti[o[r] + j] = __ldcg(p.sidx + src + j);
+        }
+      }
+    }
+    bstamp(p, 23);
   }
-  // --- window check: R < K <= R + W (W + R = n) ---
+  __syncthreads();
+  bstamp(p, 7);
+  const int n = (int)sh.cnt;
+  if (sh.bad || n > kBFcap || n < (int)p.k) {
+    fail();  // slot overflow / too many entries / fewer than K keys up to hi
+    return;
+  }
+  bstamp(p, 8);
+  const int tcnt = (n + kBBlock - 1) / kBBlock;  // entry rounds (block-uniform)
+  // --- window check: R < K <= R + W = n, R = #codes below lo ---
+  unsigned nres = 0;
+#pragma unroll 1
+  for (int e = tid; e < n; e += kBBlock) nres += (W)stc[e] < lo;
   nres = __reduce_add_sync(kFull, nres);
-  if (tid == 0) { s_tot[0] = 0; s_out = 0; }
+  if (tid == 0) {
+    sh.tot = 0;
+    sh.out = 0;
+  }
   __syncthreads();
-  if (lane == 0 && nres) atomicAdd(&s_tot[0], (unsigned long long)nres);
+  if (lane == 0 && nres) atomicAdd(&sh.tot, (unsigned long long)nres);
   __syncthreads();
-  const unsigned long long R = s_tot[0];
+  const unsigned long long R = sh.tot;
   const unsigned long long kk = (unsigned long long)p.k;
+  bstamp(p, 9);
   if (!(R < kk && kk <= (unsigned long long)n)) {
-    if (tid == 0) st->win_state = 3;
-    __syncthreads();
+    fail();
     return;
   }
   U* ov = (U*)p.out_vals + row * p.k;
@@ -357,7 +546,7 @@ __device__ void batch_finish_row(const BatchParams& p, int64_t row, void* stage)
     const unsigned m = __ballot_sync(kFull, pred);
     if (!m) return;
     unsigned b = 0;
-    if (lane == 0) b = atomicAdd(&s_out, (unsigned)__popc(m));
+    if (lane == 0) b = atomicAdd(&sh.out, (unsigned)__popc(m));
     b = __shfl_sync(kFull, b, 0);
     if (pred) {
       const unsigned pos = b + __popc(m & lanemask_lt());
@@ -365,109 +554,218 @@ __device__ void batch_finish_row(const BatchParams& p, int64_t row, void* stage)
       oi[pos] = (int64_t)idx + p.idx_off;
     }
   };
-  // results: every code below the window
-#pragma unroll
-  for (int t = 0; t < PER; ++t) {
-    const bool isr = ((valid >> t) & 1u) && (W)vc[t] < (W)lo;
-    emit(isr, vc[t], vi[t]);
-    if (isr) valid &= ~(1u << t);
+  // results (every code below the window) leave now; members stay valid; their extremes
+  unsigned valid = 0;
+  W mmin = ~(W)0, mmax = 0;
+#pragma unroll 1
+  for (int t = 0, e = tid; t < tcnt; ++t, e += kBBlock) {
+    const bool in = e < n;
+    const U c = in ? stc[e] : (U)0;
+    const bool isr = in && (W)c < lo;
+    emit(isr, c, in ? sti[e] : 0u);
+    if (in && !isr) {
+      valid |= 1u << t;
+      mmin = (W)c < mmin ? (W)c : mmin;
+      mmax = (W)c > mmax ? (W)c : mmax;
+    }
   }
-  // --- members: the K - R smallest composite keys (code || index), radix passes on registers ---
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const W a = shfl(mmin, lane ^ o), b = shfl(mmax, lane ^ o);
+    mmin = a < mmin ? a : mmin;
+    mmax = b > mmax ? b : mmax;
+  }
+  if (lane == 0) {
+    sh.wmin[warp] = mmin;
+    sh.wmax[warp] = mmax;
+  }
+  __syncthreads();
+  mmin = sh.wmin[lane];
+  mmax = sh.wmax[lane];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const W a = shfl(mmin, lane ^ o), b = shfl(mmax, lane ^ o);
+    mmin = a < mmin ? a : mmin;
+    mmax = b > mmax ? b : mmax;
+  }
+  bstamp(p, 10);
+  // --- members: the K - R smallest composite keys (code : R bits || index : IB bits), MSD radix
+  // passes of <= 11 bits starting at the highest code bit where the members differ (digits above
+  // are common to all of them); a digit never straddles the code / index boundary ---
   unsigned long long Kr = kk - R, C = (unsigned long long)n - R;
-  int q = 0;
-  const int pc = code_passes(KT<KIND>::R), P = pc + idx_passes(p.IB);
-  while (q < pc - 1) {  // digits on which lo and hi agree are common to every member
-    const Digit d = digit_of(q, KT<KIND>::R, p.IB);
-    if ((lo >> d.shift) != (hi >> d.shift)) break;
-    ++q;
-  }
-  for (; q < P && !(Kr == C && p.early_stop == 0); ++q) {
-    const Digit d = digit_of(q, KT<KIND>::R, p.IB);
-    const unsigned dm = (1u << d.width) - 1u;
-    const int nb = 1 << d.width;
-    for (int i = tid; i < nb; i += kBBlock) s_hist[i] = 0;
+  const W diff = mmin ^ mmax;
+  int pos = p.IB + (diff ? (WB - (sizeof(W) == 8 ? __clzll((long long)diff) : __clz((int)diff))) : 0);
+  int npass = 0;
+#pragma unroll 1
+  while (pos > 0 && !(Kr == C && p.early_stop == 0)) {
+    const bool is_idx = pos <= p.IB;
+    const int top = is_idx ? pos : pos - p.IB;
+    const int w = top < kDigitBits ? top : kDigitBits, shf = top - w;
+    const unsigned dm = (1u << w) - 1u;
+    for (int i = tid; i < (1 << w); i += kBBlock) sh.hist[i] = 0;
     __syncthreads();
-#pragma unroll
-    for (int t = 0; t < PER; ++t) {
+#pragma unroll 1
+    for (int t = 0, e = tid; t < tcnt; ++t, e += kBBlock) {
       if ((valid >> t) & 1u) {
-        const unsigned dg = d.is_idx ? (vi[t] >> d.shift) & dm : (unsigned)((W)vc[t] >> d.shift) & dm;
-        atomicAdd(&s_hist[dg], 1u);
+        const unsigned d = is_idx ? (sti[e] >> shf) & dm : (unsigned)((W)stc[e] >> shf) & dm;
+        atomicAdd(&sh.hist[d], 1u);
       }
     }
     __syncthreads();
-    const ScanResult r = scan_choose<kBBlock>([&](int b) { return (unsigned long long)s_hist[b]; }, nb, Kr, s_tmp,
-                                             &s_res);
-#pragma unroll
-    for (int t = 0; t < PER; ++t) {
+    const ScanResult r = scan_choose<kBBlock>([&](int b) { return (unsigned long long)sh.hist[b]; }, 1 << w, Kr,
+                                             sh.tmp, &sh.res);
+#pragma unroll 1
+    for (int t = 0, e = tid; t < tcnt; ++t, e += kBBlock) {
       const bool v = (valid >> t) & 1u;
-      const unsigned dg = d.is_idx ? (vi[t] >> d.shift) & dm : (unsigned)((W)vc[t] >> d.shift) & dm;
-      emit(v && dg < r.j, vc[t], vi[t]);
-      if (!(v && dg == r.j)) valid &= ~(1u << t);
+      const U c = v ? stc[e] : (U)0;
+      const unsigned ix = v ? sti[e] : 0u;
+      const unsigned d = is_idx ? (ix >> shf) & dm : (unsigned)((W)c >> shf) & dm;
+      emit(v && d < r.j, c, ix);
+      if (!(v && d == r.j)) valid &= ~(1u << t);
     }
     Kr -= r.before;
     C = r.cnt;
+    pos -= w;
+    bstamp(p, 11 + min(npass++, 2));
   }
-  // early stop (K == C) or the last digit: every remaining candidate is a result
-#pragma unroll
-  for (int t = 0; t < PER; ++t) emit((valid >> t) & 1u, vc[t], vi[t]);
+  // early stop (K == C, P:186) or the last digit: every remaining candidate is a result
+#pragma unroll 1
+  for (int t = 0, e = tid; t < tcnt; ++t, e += kBBlock) {
+    const bool v = (valid >> t) & 1u;
+    emit(v, v ? stc[e] : (U)0, v ? sti[e] : 0u);
+  }
   __syncthreads();
+  bstamp(p, 14);
   if (tid == 0) {
-    st->out_count = s_out;
+    st->out_count = sh.out;
     st->win_state = 4;  // done
-    if (s_out != (unsigned)kk) st->error |= 4u;
+    if (sh.out != (unsigned)kk) st->error |= 4u;
   }
+  __syncthreads();
 }
 
 template <int KIND>
 __global__ void __launch_bounds__(kBBlock, 1) batch_kernel(const BatchParams p) {
   namespace cg = cooperative_groups;
-  extern __shared__ __align__(16) unsigned char batch_smem[];
+  using U = typename KT<KIND>::U;
+  using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
+  extern __shared__ __align__(128) unsigned char batch_smem[];
+  __shared__ BatchShared<W> sh;
   cg::grid_group grid = cg::this_grid();
-  const int G = (int)gridDim.x, cta = (int)blockIdx.x;
-  auto stamp = [&](int f) {
-    if (p.timing && threadIdx.x == 0 && (int64_t)cta * 8 + f < p.timing_n) {
-      unsigned long long t;
-      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-      p.timing[(int64_t)cta * 8 + f] = (int64_t)t;
-    }
-  };
-  stamp(0);
+  const int G = (int)gridDim.x, cta = (int)blockIdx.x, tid = threadIdx.x;
+  const unsigned ring = smem_addr(batch_smem);
+  const unsigned fullb = ring + (unsigned)kBRingBytes, emptyb = fullb + 8u * kBStages;
   const int64_t nch = p.batch * (int64_t)p.cpc;
-  // L2 prefetch of the first chunks this CTA streams in phase B (overlaps the sampling latency)
-  if (threadIdx.x < 2) {
-    const int64_t ch = cta + (int64_t)threadIdx.x * G;
-    if (ch < nch) {
-      using U = typename KT<KIND>::U;
-      const int64_t row = ch / p.cpc, ci = ch % p.cpc;
-      const int64_t e0 = ci * (int64_t)kBChunkVec * (16 / sizeof(U));
-      const int64_t e1 = min(p.len, e0 + (int64_t)kBChunkVec * (16 / (int64_t)sizeof(U)));
-      prefetch_l2((const U*)p.keys + row * p.len + e0, (unsigned)((e1 - e0) * sizeof(U)));
+  const int64_t mine = cta < nch ? (nch - 1 - cta) / G + 1 : 0;  // chunks cta, cta + G, ...
+  bstamp(p, 0);
+  // the first kBPre chunks this CTA streams start landing in the ring while the rows are sampled
+  if (tid == 0) {
+    if (cta == 0) *p.fail = 0;  // (appends happen after the first grid barrier)
+    for (int i = 0; i < kBStages; ++i) {
+      mbar_init(fullb + 8u * i, 1);
+      mbar_init(emptyb + 8u * i, kBGWarps);
+    }
+    fence_mbar_init();
+    if (cta >= p.batch) {  // no row to sample: start streaming into the ring (and L2) at once
+      for (int i = 0; i < kBPre && i < mine; ++i) batch_issue<U>(p, cta + (int64_t)i * G, ring, i);
+      for (int i = kBPre; i < kBPre + kBL2Pre && i < mine; ++i) batch_prefetch_l2<U>(p, cta + (int64_t)i * G);
     }
   }
-  for (int64_t row = cta; row < p.batch; row += G) batch_sample_row<KIND>(p, row, batch_smem);
-  stamp(1);
+  __syncthreads();
+  // ---- A: windows (samples in the ring stages not yet in use); a sampling CTA issues its first
+  // bulk copies once its scattered sample loads have returned (they must not queue behind them) ----
+  for (int64_t row = cta; row < p.batch; row += G)
+    batch_sample_row<KIND>(p, row, batch_smem + kBPre * kBStage, sh, row == cta ? mine : 0, ring);
+#ifdef AIRTOPK_BATCH_TWICE  // debug: a second (warm instruction cache) sampling pass, stamps overwritten
+  for (int64_t row = cta; row < p.batch; row += G)
+    batch_sample_row<KIND>(p, row, batch_smem + kBPre * kBStage, sh, 0, ring);
+#endif
+  bstamp(p, 3);
   grid.sync();
-  stamp(2);
-  for (int64_t ch = cta; ch < nch; ch += G) {
-    const int64_t row = ch / p.cpc;
-    const int ci = (int)(ch - row * p.cpc);
-    const RowState* st = p.st + row;
-    if (st->win_state != 1) continue;
-    batch_stream_chunk<KIND>(p, row, ci, st->win_hi);
+  bstamp(p, 4);
+  // ---- B: stream every chunk once through the ring; group g consumes iterations i = g (mod 2) ----
+  if (tid == 0) {
+    fence_proxy_async_smem();  // the sample writes precede the bulk copies into the same stages
+    for (int i = kBPre; i < kBStages && i < mine; ++i) batch_issue<U>(p, cta + (int64_t)i * G, ring, i);
   }
-  stamp(3);
+  {
+    const int grp = (tid >> 5) / kBGWarps, gt = tid & (kBGThreads - 1), gw = gt >> 5;
+    const int64_t rb = p.len * (int64_t)sizeof(U);
+    // chunk cta + i*G = (row, ci), advanced incrementally by 2 iterations; the next chunk's window is
+    // loaded one iteration ahead (its L2 latency must not sit in front of every chunk)
+    const int64_t step = (int64_t)kBGroups * G;
+    const int64_t drow = step / p.cpc;
+    const int dci = (int)(step - drow * p.cpc);
+    const int64_t ch0 = cta + (int64_t)grp * G;
+    int64_t row = ch0 / p.cpc;
+    int ci = (int)(ch0 - row * p.cpc);
+    int ws = 0;
+    unsigned long long hi = 0;
+    if (grp < mine) {
+      ws = p.st[row].win_state;
+      hi = p.st[row].win_hi;
+    }
+    int st = grp;
+    unsigned ph = 0;
+#pragma unroll 1
+    for (int64_t i = grp; i < mine; i += kBGroups) {
+      int64_t nrow = row + drow;
+      int nci = ci + dci;
+      if (nci >= p.cpc) {
+        nci -= p.cpc;
+        ++nrow;
+      }
+      int nws = 0;
+      unsigned long long nhi = 0;
+      if (i + kBGroups < mine) {
+        nws = p.st[nrow].win_state;
+        nhi = p.st[nrow].win_hi;
+      }
+      const int64_t left = rb - ci * (int64_t)kBStage;
+      mbar_wait_sleep(fullb + 8u * st, ph);
+      if (ws == 1) {
+        if (left >= (int64_t)kBStage) batch_classify<KIND, true>(p, row, ci, hi, ring + st * kBStage, 0, gt, gw);
+        else batch_classify<KIND, false>(p, row, ci, hi, ring + st * kBStage, (int)(left / 16), gt, gw);
+      }
+      __syncwarp();
+      if ((tid & 31) == 0) mbar_arrive(emptyb + 8u * st);
+      // the group leader refills the stage with the chunk kBStages iterations ahead
+      if (gt == 0 && i + kBStages < mine) {
+        mbar_wait_sleep(emptyb + 8u * st, ph);
+        fence_proxy_async_smem();
+        batch_issue<U>(p, cta + (i + kBStages) * G, ring, st);
+      }
+      st += kBGroups;
+      if (st >= kBStages) {
+        st -= kBStages;
+        ph ^= 1u;
+      }
+      row = nrow;
+      ci = nci;
+      ws = nws;
+      hi = nhi;
+    }
+  }
+  bstamp(p, 5);
+  // touch the pages phase C reads first (slot counts and entries of this CTA's first row): their
+  // address translations are then cached before the barrier instead of after it
+  if (tid < 3 && cta < p.batch) {
+    const char* a = tid == 0 ? (const char*)(p.cnt + (size_t)cta * p.nwc)
+                  : tid == 1 ? (const char*)p.scode + (size_t)cta * p.nwc * p.scap * sizeof(U)
+                             : (const char*)(p.sidx + (size_t)cta * p.nwc * p.scap);
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(a) : "memory");
+  }
   grid.sync();
-  stamp(4);
-  for (int64_t row = cta; row < p.batch; row += G) batch_finish_row<KIND>(p, row, batch_smem);
-  stamp(5);
+  bstamp(p, 6);
+  // ---- C: finish every row (staging in the ring: every bulk copy has been consumed) ----
+  for (int64_t row = cta; row < p.batch; row += G) batch_finish_row<KIND>(p, row, batch_smem, sh);
+  bstamp(p, 15);
 }
 
 template <int KIND>
 constexpr size_t batch_smem_bytes() {
-  using U = typename KT<KIND>::U;
-  const size_t fin = (size_t)batch_fcap<KIND>() * (sizeof(U) + 4);
-  const size_t samp = (size_t)kMaxSamples * (sizeof(U) == 8 ? 8 : 4);
-  return fin > samp ? fin : samp;
+  static_assert((size_t)kBFcap * (sizeof(typename KT<KIND>::U) + 4) <= kBRingBytes, "finish staging fits the ring");
+  return kBRingBytes + 16 * kBStages;
 }
 
 template <int KIND>
@@ -482,8 +780,11 @@ cudaError_t launch_batch_kind(const SelectArgs& a, const Plan& pl, void* ws, cud
   cudaError_t e = func_attr(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int occ = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBBlock, smem);
-  if (e != cudaSuccess) return e;
+  if (!occ_cache_get((const void*)kern, 0, &occ)) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBBlock, smem);
+    if (e != cudaSuccess) return e;
+    occ_cache_put((const void*)kern, 0, occ);
+  }
   if (occ < 1) return cudaErrorInvalidConfiguration;
   char* base = (char*)ws;
   BatchParams p;
@@ -500,6 +801,7 @@ cudaError_t launch_batch_kind(const SelectArgs& a, const Plan& pl, void* ws, cud
   p.cnt = (unsigned short*)(base + pl.off_bcnt);
   p.scode = base + pl.off_bslot;
   p.sidx = (unsigned*)(base + pl.off_bsidx);
+  p.fail = (unsigned*)(base + pl.off_bfail);
   p.nwc = pl.nwc;
   p.scap = pl.scap;
   p.cpc = pl.cpc;

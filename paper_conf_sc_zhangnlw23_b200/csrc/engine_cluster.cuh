@@ -51,6 +51,7 @@ struct ClusterParams {
   int tail_q;    // tail mode: the grid engine ran passes q < tail_q after the window pass
   int timing_stride;  // int64 slots per CTA in `timing` (8; 24 with the merge-phase stamps, debug)
   int64_t* timing;  // optional: per CTA [globaltimer at start, at end, rows done, passes run, end of passes 1-4]
+  const unsigned* fail;  // tail == 2: [0] = number of rows to redo, [1 + i] = the rows
 };
 
 struct ClusterShared {
@@ -101,9 +102,10 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
     }
   };
 
-  for (int64_t row = cid; row < p.batch; row += p.nclusters) {
+  const int64_t nrows = (p.tail == 2) ? (int64_t)p.fail[0] : p.batch;  // fallback: only the failed rows
+  for (int64_t it = cid; it < nrows; it += p.nclusters) {
+    const int64_t row = (p.tail == 2) ? (int64_t)p.fail[1 + it] : it;
     RowState* st = p.st + row;
-    if (p.tail == 2 && st->win_state != 3) continue;  // (cluster-uniform) finished by the batched engine
     unsigned long long K = kk, C = N, Cp = N, tcode = 0, tidx = 0;
     int stop1 = 0, src1 = 0;  // src1: 0 = the input row L, s + 1 = candidate buffer slot s
     int q0 = 0;
@@ -313,6 +315,7 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   // standalone cluster engine: the trace buffer receives per-CTA timing instead (not in tail /
   // fallback mode: the trace then belongs to the engine that ran before)
   p.timing = tail ? nullptr : a.trace;
+  p.fail = (const unsigned*)(base + pl.off_bfail);
   p.timing_stride = getenv("AIRTOPK_CLUSTER_TIMING") ? 24 : 8;
 
   cudaLaunchConfig_t cfg = {};
@@ -330,8 +333,11 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   cfg.numAttrs = tail ? 2 : 1;
   cfg.gridDim = dim3((unsigned)pl.csize, 1, 1);
   int maxc = 0;
-  e = cudaOccupancyMaxActiveClusters(&maxc, kern, &cfg);
-  if (e != cudaSuccess) return e;
+  if (!occ_cache_get((const void*)kern, pl.csize * 4 + (tail ? 1 : 0), &maxc)) {
+    e = cudaOccupancyMaxActiveClusters(&maxc, kern, &cfg);
+    if (e != cudaSuccess) return e;
+    occ_cache_put((const void*)kern, pl.csize * 4 + (tail ? 1 : 0), maxc);
+  }
   if (maxc < 1) return cudaErrorInvalidConfiguration;
   const int64_t ncl = std::min<int64_t>(a.batch, (int64_t)maxc);
   p.nclusters = (int)ncl;

@@ -379,10 +379,14 @@ constexpr int kBrute = 128;
 constexpr int kSampleHistCopies = 4;
 static_assert(kSampleBlock / 8 >= kBrute, "8 threads per bin member in the brute-force rank");
 
-template <typename W, int PER>
+struct NoStamp {
+  __device__ void operator()(int) const {}
+};
+
+template <typename W, int PER, typename Stamp = NoStamp>
 __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo, int rhi, W pmin, int hb,
                                  unsigned* hist /* 2048 x copies */, unsigned* wsum /* 32 */, W* shw, int* cnt,
-                                 W& lo, W& hi) {
+                                 W& lo, W& hi, Stamp stamp = Stamp()) {
   constexpr int WB = 8 * (int)sizeof(W);
   if (hb <= 0) {  // all samples equal
     lo = hi = pmin;
@@ -403,6 +407,7 @@ __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo,
   for (int t = 0; t < PER; ++t)
     if (t < tv) atomicAdd(&hist[((unsigned)(v[t] >> sh) & dmask) * kSampleHistCopies + hcopy], 1u);
   __syncthreads();
+  stamp(0);
   auto binc = [&](unsigned b) {
     unsigned x = 0;
 #pragma unroll
@@ -438,6 +443,7 @@ __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo,
   const unsigned blo = (rlo >= 0) ? (unsigned)shw[0] : 0xffffffffu, bhi = (unsigned)shw[1];
   const int rk_lo = rlo - (int)shw[2], rk_hi = rhi - (int)shw[3];
   const int m_lo = (rlo >= 0) ? (int)binc(blo) : 0, m_hi = (int)binc(bhi);
+  stamp(1);
   const W plo = prefix | ((W)blo << sh), phi = prefix | ((W)bhi << sh);
   if (sh == 0) {
     lo = plo;
@@ -478,6 +484,7 @@ __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo,
     }
   }
   __syncthreads();
+  stamp(2);
   // exact rank inside a bin
   const W sub = (W)dmask << sh;
   W res[2] = {plo, phi};
@@ -511,6 +518,7 @@ __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo,
       select_digits<W>(reg, m, rk, pre, msk, sh, 0, hist, shw + 6);
       res[q] = pre;
     }
+    stamp(3 + q);
   }
   lo = res[0];
   hi = res[1];

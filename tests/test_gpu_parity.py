@@ -313,13 +313,14 @@ def test_window_fallback(case, engine):
 @pytest.mark.parametrize("dist,batch,n,k", [("normal", 100, 1 << 20, 256), ("adversarial", 3, 1 << 22, 5000),
                                             ("uniform", 7, 1 << 19, 1), ("uniform", 2, 1 << 21, 20000)])
 def test_window_tail(dist, batch, n, k):
-    """auto engine: window pass + one cluster-engine launch finishing every row (tail mode)"""
+    """grid engine window pass + one cluster-engine launch finishing every row (tail mode; AUTO
+    sends batches to the batched engine, window=1 asks for the grid engine's window pass)"""
     import torch
     import paper_conf_sc_zhangnlw23_b200 as at
-    assert at.describe(torch.float32, batch, n, k)["launches"] == 3
+    assert at.describe(torch.float32, batch, n, k, window=1)["launches"] == 3
     x = _keys(dist, 33, batch, n)
     for sm in (True, False):
-        v, i = gpu_select(x, "f32", k, sm)
+        v, i = gpu_select(x, "f32", k, sm, window=1)
         assert_parity(x, "f32", k, sm, v, i)
 
 
