@@ -37,18 +37,20 @@ cudaError_t func_attr(const void* f, cudaFuncAttribute attr, int value) {
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
-  using Key = std::tuple<const void*, int, int, int>;
+  // the attribute holds ONE value per (kernel, device): remember the value last set, re-set on change
+  using Key = std::tuple<const void*, int, int>;
   static std::mutex mu;
-  static std::set<Key> done;
-  const Key key{f, dev, (int)attr, value};
+  static std::map<Key, int> cur;
+  const Key key{f, dev, (int)attr};
   {
     std::lock_guard<std::mutex> g(mu);
-    if (done.count(key)) return cudaSuccess;
+    auto it = cur.find(key);
+    if (it != cur.end() && it->second == value) return cudaSuccess;
   }
   e = cudaFuncSetAttribute(f, attr, value);
   if (e == cudaSuccess) {
     std::lock_guard<std::mutex> g(mu);
-    done.insert(key);
+    cur[key] = value;
   }
   return e;
 }
@@ -180,14 +182,15 @@ Plan make_plan(const SelectArgs& a) {
 // and small rows, the grid engine (one launch per pass, whole GPU per row) for long rows.
 static int auto_engine(const SelectArgs& a) {
   if (a.window > 0 && !a.in_idx) return 1;  // window requested: grid window pass (+ cluster tail)
-  if (a.len <= (int64_t(1) << 17)) return 2;
-  if (a.len <= (int64_t(1) << 22) && a.batch >= 16 && getenv("AIRTOPK_CLUSTER_BATCHED")) return 2;
+  if (a.len <= (int64_t(1) << 19)) return 2;  // one launch: measured fastest from 2^17 to 2^19 keys per row
   return 1;
 }
 
 static int auto_cluster_size(const SelectArgs& a) {
   if (a.cluster_size > 0) return a.cluster_size;
   int64_t c = (a.len + 4095) / 4096;  // >= 4096 elements per CTA
+  // batches: no more CTAs per row than keep every row of a wave resident (rows run concurrently)
+  if (a.batch > 1) c = std::min<int64_t>(c, std::max<int64_t>(1, (int64_t)num_sms() / a.batch));
   int cs = 1;
   while (cs < 16 && cs < c) cs <<= 1;
   return cs;
@@ -199,8 +202,37 @@ static bool batch_aligned(const SelectArgs& a) {
   return ((uintptr_t)a.keys % 16) == 0 && ((size_t)a.len * key_bytes(a.kind)) % 16 == 0;
 }
 
+// Resident-cluster engine: rows held in shared memory (a cluster of CS CTAs, <= kResidentCap keys
+// each). CS: enough CTAs to hold the row; for latency ~8K keys per CTA while the batch leaves SMs free.
+static bool resident_fits(const SelectArgs& a) {
+  const int64_t cap = key_bytes(a.kind) == 8 ? kResidentCap / 2 : kResidentCap;
+  return !a.in_idx && a.len <= 16 * cap && a.len < (int64_t(1) << 31);
+}
+
+static void resident_geometry(const SelectArgs& a, Plan& p) {
+  const int64_t cap = key_bytes(a.kind) == 8 ? kResidentCap / 2 : kResidentCap;
+  auto pow2ceil = [](int64_t v) { int64_t c = 1; while (c < v) c <<= 1; return c; };
+  const int64_t cmin = pow2ceil((a.len + cap - 1) / cap);
+  int64_t clat = pow2ceil((a.len + 8191) / 8192);
+  clat = std::min<int64_t>(clat, std::max<int64_t>(1, (int64_t)num_sms() / a.batch));
+  int64_t cs = std::min<int64_t>(16, std::max(cmin, clat));
+  if (a.cluster_size > 0) cs = std::max<int64_t>(cmin, a.cluster_size);
+  p.csize = (int)cs;
+  p.rslice = (int)(((a.len + cs - 1) / cs + 7) / 8 * 8);
+}
+
 static void choose_launch(const SelectArgs& a, Plan& p) {
   if (p.engine == 3 || p.engine == 4) return;
+  // AUTO (tools/engine_ab.py, profiles/r02_engine_ab.txt, L2 flushed between selects): the
+  // resident cluster wins for rows of <= 2^14 keys at any batch and for a single row of <= 2^16
+  if (a.engine == 6 || (a.engine == 0 && a.window == 0 && resident_fits(a) && a.trace == nullptr &&
+                        (a.len <= (int64_t(1) << 14) || (a.batch == 1 && a.len <= (int64_t(1) << 16))))) {
+    if (resident_fits(a)) {
+      p.engine = 6;
+      resident_geometry(a, p);
+      return;
+    }
+  }
   // batched engine: explicit, or AUTO for batches with enough 64 KiB chunks to cover the SMs
   if (p.batch_ok && batch_aligned(a) && (a.trace == nullptr || a.engine == 5) &&
       (a.engine == 5 || (a.engine == 0 && a.window == 0 && a.batch >= 2 && (int64_t)a.batch * p.cpc >= num_sms()))) {
@@ -209,11 +241,15 @@ static void choose_launch(const SelectArgs& a, Plan& p) {
     p.nsamp = p.bnsamp;
     return;
   }
-  p.engine = a.engine > 0 && a.engine != 5 ? a.engine : auto_engine(a);
+  p.engine = a.engine > 0 && a.engine != 5 && a.engine != 6 ? a.engine : auto_engine(a);
   if (p.engine == 2) {
     p.csize = auto_cluster_size(a);
     return;
   }
+  // rows of fewer than 2^26 keys: the sample + window (+ tail) launches cost more than the second
+  // read of L they save (tools/engine_ab.py: 1 x 2^22 keys 36 us without vs 51 us with the window,
+  // 1 x 2^24 63 vs 73 us, 100 x 2^20 with K = 32768 334 vs 723 us); the paper's passes run instead
+  if (a.window == 0 && a.engine == 0 && a.len < (int64_t(1) << 26) && !a.in_idx) p.nsamp = 0;
   // expected window size per row (entries) -> tail mode for small windows
   p.tail = 0;
   if (p.nsamp > 0 && a.window >= 0) {
@@ -265,7 +301,7 @@ static airtopk_status validate(const SelectArgs& a) {
   if (!a.keys || !a.out_vals || !a.out_idx) return AIRTOPK_EINVAL;
   if (a.batch < 1 || a.len < 1 || a.k < 1 || a.k > a.len) return AIRTOPK_EINVAL;
   if (a.alpha < 0) return AIRTOPK_EINVAL;
-  if (a.engine < 0 || a.engine > 5 || a.engine == 3) return AIRTOPK_EINVAL;
+  if (a.engine < 0 || a.engine > 6 || a.engine == 3) return AIRTOPK_EINVAL;
   if (a.engine == 4 && !gridselect_supported(a)) return AIRTOPK_EINVAL;
   if (a.window < -1 || a.window > 1) return AIRTOPK_EINVAL;
   if (a.early_stop < -1 || a.early_stop > 0) return AIRTOPK_EINVAL;
@@ -301,10 +337,12 @@ static airtopk_status run(const SelectArgs& a, void* ws, size_t ws_bytes, cudaSt
     return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
   }
   choose_launch(a, p);
+  if ((a.engine == 5 || a.engine == 6) && p.engine != a.engine) return AIRTOPK_EINVAL;  // shape not eligible
   if (p.engine == 2 && (p.csize < 1 || p.csize > 16 || (p.csize & (p.csize - 1)))) return AIRTOPK_EINVAL;
-  if (a.engine == 5 && p.engine != 5) return AIRTOPK_EINVAL;  // batched engine requested, shape not eligible
-  cudaError_t e = (p.engine == 2) ? run_cluster(a, p, ws, s) : (p.engine == 5) ? run_batch(a, p, ws, s)
-                                                                               : run_grid(a, p, ws, s);
+  cudaError_t e = (p.engine == 2)   ? run_cluster(a, p, ws, s)
+                  : (p.engine == 5) ? run_batch(a, p, ws, s)
+                  : (p.engine == 6) ? run_resident(a, p, ws, s)
+                                    : run_grid(a, p, ws, s);
   if (e == cudaSuccess && a.status) e = collect_status(a, p, ws, s);
   return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
 }
@@ -538,10 +576,10 @@ airtopk_status airtopk_describe(airtopk_dtype dtype, int64_t batch, int64_t len,
   std::memset(out, 0, sizeof(*out));
   out->engine = p.engine;
   out->passes = p.P;
-  out->launches = (p.engine == 3 || p.engine == 4) ? 1 : (p.engine == 2 ? 1 : p.engine == 5 ? 2
+  out->launches = (p.engine == 3 || p.engine == 4 || p.engine == 6) ? 1 : (p.engine == 2 ? 1 : p.engine == 5 ? 2
                   : (p.tail ? 3 + p.tail_q : p.P + 1 + (p.nsamp > 0 ? 2 : 0)));
   out->ctas_per_row = (p.engine == 1 || p.engine == 4) ? p.cpr : 0;
-  out->cluster_size = (p.engine == 2 || p.engine == 5 || p.tail) ? p.csize : 0;
+  out->cluster_size = (p.engine == 2 || p.engine == 5 || p.engine == 6 || p.tail) ? p.csize : 0;
   out->index_bits = p.IB;
   out->buffer_cap = p.cap_rule;
   out->workspace_bytes = bytes;

@@ -32,7 +32,7 @@ struct SelectArgs {
 
 // Resolved launch plan (host side).
 struct Plan {
-  int engine;        // 1 grid, 2 cluster, 3 trivial copy (K == N), 4 GridSelect
+  int engine;        // 1 grid, 2 cluster, 3 trivial copy (K == N), 4 GridSelect, 5 batched, 6 resident cluster
   int idx64;         // 64-bit internal indices
   int R;             // key bits
   int IB;            // index bits appended to the key for the lowest-index tie-break
@@ -53,6 +53,7 @@ struct Plan {
   int cpc;           // 32 KiB chunks per row
   int nwc;           // (chunk, warp) slots per row
   int scap;          // entries per slot
+  int rslice;        // resident-cluster engine: keys per CTA
   size_t off_state, off_hist, off_bcode, off_bidx, off_samp, off_bcnt, off_bslot, off_bsidx, off_bfail, bytes;
 };
 
@@ -76,11 +77,15 @@ Plan make_plan(const SelectArgs& a);
 cudaError_t run_grid(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 cudaError_t run_cluster(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 cudaError_t run_batch(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
+cudaError_t run_resident(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 // batched engine constants shared with the host plan (engine_batch.cuh)
 constexpr int kBatchBlock = 1024, kBatchWarps = 32;
 constexpr int kBatchSlotWarps = 16;  // warps per consumer group = (chunk, warp) slots per chunk
 constexpr int kBatchStage = 32768;   // bytes per chunk (one bulk-copy ring stage)
 constexpr int kBatchFcap = 16384;    // entries (results + window members) one row may stage in the finish
+// resident-cluster engine (engine_resident.cuh)
+constexpr int kResidentCap = 32768;  // keys per CTA held in shared memory (<= 4-byte keys; half for 8-byte)
+constexpr int kResidentFin = 2048;   // candidates CTA 0 finishes
 cudaError_t run_trivial(const SelectArgs& a, cudaStream_t s);
 // K entries that sort last in the selection order (multi-GPU shard shorter than K): value bits of the
 // maximum code, indices pad_base + j

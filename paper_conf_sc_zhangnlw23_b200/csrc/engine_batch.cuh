@@ -41,6 +41,7 @@
 #include "device.cuh"
 #include "engine.h"
 #include "engine_grid.cuh"
+#include "finish.cuh"
 #include "tma.cuh"
 
 namespace airtopk {
@@ -108,6 +109,7 @@ struct BatchShared {
   unsigned long long tmp[kBWarps];
   ScanResult res;
   W wmin[kBWarps], wmax[kBWarps];
+  SelScratch<W, kBWarps> sel;   // finish: shared-memory radix select
   W result;
   unsigned long long tot;
   unsigned cnt, out;
@@ -554,86 +556,20 @@ __device__ void batch_finish_row(const BatchParams& p, int64_t row, void* stage,
       oi[pos] = (int64_t)idx + p.idx_off;
     }
   };
-  // results (every code below the window) leave now; members stay valid; their extremes
+  // results (every code below the window) leave now; members stay live
   unsigned valid = 0;
-  W mmin = ~(W)0, mmax = 0;
 #pragma unroll 1
   for (int t = 0, e = tid; t < tcnt; ++t, e += kBBlock) {
     const bool in = e < n;
     const U c = in ? stc[e] : (U)0;
     const bool isr = in && (W)c < lo;
     emit(isr, c, in ? sti[e] : 0u);
-    if (in && !isr) {
-      valid |= 1u << t;
-      mmin = (W)c < mmin ? (W)c : mmin;
-      mmax = (W)c > mmax ? (W)c : mmax;
-    }
-  }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    const W a = shfl(mmin, lane ^ o), b = shfl(mmax, lane ^ o);
-    mmin = a < mmin ? a : mmin;
-    mmax = b > mmax ? b : mmax;
-  }
-  if (lane == 0) {
-    sh.wmin[warp] = mmin;
-    sh.wmax[warp] = mmax;
-  }
-  __syncthreads();
-  mmin = sh.wmin[lane];
-  mmax = sh.wmax[lane];
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    const W a = shfl(mmin, lane ^ o), b = shfl(mmax, lane ^ o);
-    mmin = a < mmin ? a : mmin;
-    mmax = b > mmax ? b : mmax;
+    if (in && !isr) valid |= 1u << t;
   }
   bstamp(p, 10);
-  // --- members: the K - R smallest composite keys (code : R bits || index : IB bits), MSD radix
-  // passes of <= 11 bits starting at the highest code bit where the members differ (digits above
-  // are common to all of them); a digit never straddles the code / index boundary ---
-  unsigned long long Kr = kk - R, C = (unsigned long long)n - R;
-  const W diff = mmin ^ mmax;
-  int pos = p.IB + (diff ? (WB - (sizeof(W) == 8 ? __clzll((long long)diff) : __clz((int)diff))) : 0);
-  int npass = 0;
-#pragma unroll 1
-  while (pos > 0 && !(Kr == C && p.early_stop == 0)) {
-    const bool is_idx = pos <= p.IB;
-    const int top = is_idx ? pos : pos - p.IB;
-    const int w = top < kDigitBits ? top : kDigitBits, shf = top - w;
-    const unsigned dm = (1u << w) - 1u;
-    for (int i = tid; i < (1 << w); i += kBBlock) sh.hist[i] = 0;
-    __syncthreads();
-#pragma unroll 1
-    for (int t = 0, e = tid; t < tcnt; ++t, e += kBBlock) {
-      if ((valid >> t) & 1u) {
-        const unsigned d = is_idx ? (sti[e] >> shf) & dm : (unsigned)((W)stc[e] >> shf) & dm;
-        atomicAdd(&sh.hist[d], 1u);
-      }
-    }
-    __syncthreads();
-    const ScanResult r = scan_choose<kBBlock>([&](int b) { return (unsigned long long)sh.hist[b]; }, 1 << w, Kr,
-                                             sh.tmp, &sh.res);
-#pragma unroll 1
-    for (int t = 0, e = tid; t < tcnt; ++t, e += kBBlock) {
-      const bool v = (valid >> t) & 1u;
-      const U c = v ? stc[e] : (U)0;
-      const unsigned ix = v ? sti[e] : 0u;
-      const unsigned d = is_idx ? (ix >> shf) & dm : (unsigned)((W)c >> shf) & dm;
-      emit(v && d < r.j, c, ix);
-      if (!(v && d == r.j)) valid &= ~(1u << t);
-    }
-    Kr -= r.before;
-    C = r.cnt;
-    pos -= w;
-    bstamp(p, 11 + min(npass++, 2));
-  }
-  // early stop (K == C) or the last digit: every remaining candidate is a result
-#pragma unroll 1
-  for (int t = 0, e = tid; t < tcnt; ++t, e += kBBlock) {
-    const bool v = (valid >> t) & 1u;
-    emit(v, v ? stc[e] : (U)0, v ? sti[e] : 0u);
-  }
+  // members: the K - R smallest composite keys (code || index), radix passes in shared memory
+  block_select_smem<KIND, kBBlock>(stc, sti, tcnt, valid, kk - R, (unsigned long long)n - R, p.IB,
+                                   p.early_stop == 0, sh.sel, emit);
   __syncthreads();
   bstamp(p, 14);
   if (tid == 0) {

@@ -1,5 +1,6 @@
 // Grid- and cluster-engine kernels instantiated for key type F16 (see engine_grid.cuh).
 #include "engine_batch.cuh"
+#include "engine_resident.cuh"
 #include "engine_cluster.cuh"
 #include "engine_grid.cuh"
 
@@ -7,4 +8,5 @@ namespace airtopk {
 AIRTOPK_INSTANTIATE_GRID(K_F16)
 AIRTOPK_INSTANTIATE_CLUSTER(K_F16)
 AIRTOPK_INSTANTIATE_BATCH(K_F16)
+AIRTOPK_INSTANTIATE_RESIDENT(K_F16)
 }  // namespace airtopk

@@ -1,5 +1,6 @@
 // Grid- and cluster-engine kernels instantiated for key type F32 (see engine_grid.cuh).
 #include "engine_batch.cuh"
+#include "engine_resident.cuh"
 #include "engine_cluster.cuh"
 #include "engine_grid.cuh"
 
@@ -7,6 +8,7 @@ namespace airtopk {
 AIRTOPK_INSTANTIATE_GRID(K_F32)
 AIRTOPK_INSTANTIATE_CLUSTER(K_F32)
 AIRTOPK_INSTANTIATE_BATCH(K_F32)
+AIRTOPK_INSTANTIATE_RESIDENT(K_F32)
 
 int grid_occupancy_f32(int idx64) {
   int n = 0;

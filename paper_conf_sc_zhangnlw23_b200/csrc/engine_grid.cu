@@ -2,6 +2,7 @@
 // K == N trivial path. The kernels live in engine_grid.cuh and are instantiated per key type in
 // engine_grid_<kind>.cu (parallel compilation).
 #include "engine_batch.cuh"
+#include "engine_resident.cuh"
 #include "engine_cluster.cuh"
 #include "engine_grid.cuh"
 
@@ -16,10 +17,15 @@ extern template cudaError_t launch_grid_kind<K_F64>(const SelectArgs&, const Pla
 extern template cudaError_t launch_grid_kind<K_U32>(const SelectArgs&, const Plan&, const GridParams&, void*, cudaStream_t);
 int grid_occupancy_f32(int idx64);
 extern template cudaError_t launch_batch_kind<K_F32>(const SelectArgs&, const Plan&, void*, cudaStream_t);
+extern template cudaError_t launch_resident_kind<K_F32>(const SelectArgs&, const Plan&, void*, cudaStream_t);
 extern template cudaError_t launch_batch_kind<K_F16>(const SelectArgs&, const Plan&, void*, cudaStream_t);
+extern template cudaError_t launch_resident_kind<K_F16>(const SelectArgs&, const Plan&, void*, cudaStream_t);
 extern template cudaError_t launch_batch_kind<K_BF16>(const SelectArgs&, const Plan&, void*, cudaStream_t);
+extern template cudaError_t launch_resident_kind<K_BF16>(const SelectArgs&, const Plan&, void*, cudaStream_t);
 extern template cudaError_t launch_batch_kind<K_F64>(const SelectArgs&, const Plan&, void*, cudaStream_t);
+extern template cudaError_t launch_resident_kind<K_F64>(const SelectArgs&, const Plan&, void*, cudaStream_t);
 extern template cudaError_t launch_batch_kind<K_U32>(const SelectArgs&, const Plan&, void*, cudaStream_t);
+extern template cudaError_t launch_resident_kind<K_U32>(const SelectArgs&, const Plan&, void*, cudaStream_t);
 extern template cudaError_t launch_cluster_kind<K_F32>(const SelectArgs&, const Plan&, void*, cudaStream_t, int);
 extern template cudaError_t launch_cluster_kind<K_F16>(const SelectArgs&, const Plan&, void*, cudaStream_t, int);
 extern template cudaError_t launch_cluster_kind<K_BF16>(const SelectArgs&, const Plan&, void*, cudaStream_t, int);
@@ -92,6 +98,18 @@ cudaError_t run_batch(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_
     case K_BF16: return launch_batch_kind<K_BF16>(a, pl, ws, s);
     case K_F64: return launch_batch_kind<K_F64>(a, pl, ws, s);
     case K_U32: return launch_batch_kind<K_U32>(a, pl, ws, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+cudaError_t run_resident(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t s) {
+  // (no memset: the kernel resets each row's counters itself)
+  switch (a.kind) {
+    case K_F32: return launch_resident_kind<K_F32>(a, pl, ws, s);
+    case K_F16: return launch_resident_kind<K_F16>(a, pl, ws, s);
+    case K_BF16: return launch_resident_kind<K_BF16>(a, pl, ws, s);
+    case K_F64: return launch_resident_kind<K_F64>(a, pl, ws, s);
+    case K_U32: return launch_resident_kind<K_U32>(a, pl, ws, s);
   }
   return cudaErrorInvalidValue;
 }

@@ -1,0 +1,128 @@
+// finish.cuh — single-CTA selection over a small candidate set held in shared memory.
+//
+// The last step of a row once its candidates fit one CTA (the batched engine's per-row finish, the
+// resident-cluster engine's small finish): among n (code, index) entries, the Kr smallest composite
+// keys (code : R bits || index : IB bits — the lowest-index tie rule, reading 1) are
+// emitted. It is the paper's radix select (Alg1 L15-28) on shared memory: per pass a
+// histogram of one <= 11-bit digit, the inclusive scan and the target digit j with
+// psum[j-1] < K <= psum[j], the filter (digit < j -> result, == j -> candidate), early stop when
+// K == C. Passes start at the highest code bit where the entries differ (the digits above
+// are common to all of them, their histograms would be single bins); a digit never straddles the
+// code / index boundary. Code is compact (rolled loops): it runs once per row on a cold
+// instruction cache.
+#pragma once
+
+#include "device.cuh"
+
+namespace airtopk {
+
+template <typename W, int NW>
+struct SelScratch {
+  unsigned hist[kMaxBins];
+  unsigned long long tmp[NW];
+  ScanResult res;
+  W wmin[NW], wmax[NW];
+};
+
+// Entry e = tid + t * BLOCK (t < tcnt, block-uniform) is live iff bit t of `valid`. C = number of
+// live entries (block-wide), Kr <= C. emit(pred, code, idx) is called by every thread (warp
+// collective) for each of its slots; it must place the selected entries.
+template <int KIND, int BLOCK, typename Emit>
+__device__ void block_select_smem(const typename KT<KIND>::U* stc, const unsigned* sti, int tcnt, unsigned valid,
+                                  unsigned long long Kr, unsigned long long C, int IB, bool early_stop,
+                                  SelScratch<std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long,
+                                                                unsigned>, BLOCK / 32>& sh,
+                                  Emit emit) {
+  using U = typename KT<KIND>::U;
+  using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
+  constexpr int WB = 8 * (int)sizeof(W);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (C <= 32 && tcnt == 1 && __syncthreads_and(tid < 32 || !(valid & 1u))) {
+    // at most 32 live entries, all held by warp 0: rank them by counting (one shuffle round) — the
+    // K smallest composite keys are the ranks < K (keys are unique)
+    if (warp == 0) {
+      const bool v = valid & 1u;
+      const U c = v ? stc[tid] : (U)0;
+      const unsigned ix = v ? sti[tid] : 0u;
+      unsigned rank = 0;
+      for (int o = 0; o < 32; ++o) {
+        const bool vo = __shfl_sync(kFull, (int)v, o);
+        const W co = (W)shfl((W)c, o);
+        const unsigned io = __shfl_sync(kFull, ix, o);
+        rank += vo && (co < (W)c || (co == (W)c && io < ix));
+      }
+      emit(v && rank < Kr, c, ix);
+    }
+    return;
+  }
+  // extremes of the live codes: the digits above their highest differing bit are common
+  W mmin = ~(W)0, mmax = 0;
+#pragma unroll 1
+  for (int t = 0, e = tid; t < tcnt; ++t, e += BLOCK) {
+    if ((valid >> t) & 1u) {
+      const W c = (W)stc[e];
+      mmin = c < mmin ? c : mmin;
+      mmax = c > mmax ? c : mmax;
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const W a = shfl(mmin, lane ^ o), b = shfl(mmax, lane ^ o);
+    mmin = a < mmin ? a : mmin;
+    mmax = b > mmax ? b : mmax;
+  }
+  if (lane == 0) {
+    sh.wmin[warp] = mmin;
+    sh.wmax[warp] = mmax;
+  }
+  __syncthreads();
+  mmin = lane < BLOCK / 32 ? sh.wmin[lane] : ~(W)0;
+  mmax = lane < BLOCK / 32 ? sh.wmax[lane] : (W)0;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const W a = shfl(mmin, lane ^ o), b = shfl(mmax, lane ^ o);
+    mmin = a < mmin ? a : mmin;
+    mmax = b > mmax ? b : mmax;
+  }
+  const W diff = mmin ^ mmax;
+  int pos = IB + (diff ? (WB - (sizeof(W) == 8 ? __clzll((long long)diff) : __clz((int)diff))) : 0);
+#pragma unroll 1
+  while (pos > 0 && !(Kr == C && early_stop)) {
+    const bool is_idx = pos <= IB;
+    const int top = is_idx ? pos : pos - IB;
+    const int w = top < kDigitBits ? top : kDigitBits, shf = top - w;
+    const unsigned dm = (1u << w) - 1u;
+    for (int i = tid; i < (1 << w); i += BLOCK) sh.hist[i] = 0;
+    __syncthreads();
+#pragma unroll 1
+    for (int t = 0, e = tid; t < tcnt; ++t, e += BLOCK) {
+      if ((valid >> t) & 1u) {
+        const unsigned d = is_idx ? (sti[e] >> shf) & dm : (unsigned)((W)stc[e] >> shf) & dm;
+        atomicAdd(&sh.hist[d], 1u);
+      }
+    }
+    __syncthreads();
+    const ScanResult r = scan_choose<BLOCK>([&](int b) { return (unsigned long long)sh.hist[b]; }, 1 << w, Kr,
+                                           sh.tmp, &sh.res);
+#pragma unroll 1
+    for (int t = 0, e = tid; t < tcnt; ++t, e += BLOCK) {
+      const bool v = (valid >> t) & 1u;
+      const U c = v ? stc[e] : (U)0;
+      const unsigned ix = v ? sti[e] : 0u;
+      const unsigned d = is_idx ? (ix >> shf) & dm : (unsigned)((W)c >> shf) & dm;
+      emit(v && d < r.j, c, ix);
+      if (!(v && d == r.j)) valid &= ~(1u << t);
+    }
+    Kr -= r.before;
+    C = r.cnt;
+    pos -= w;
+  }
+  // early stop (K == C) or the last digit: every remaining candidate is a result
+#pragma unroll 1
+  for (int t = 0, e = tid; t < tcnt; ++t, e += BLOCK) {
+    const bool v = (valid >> t) & 1u;
+    emit(v, v ? stc[e] : (U)0, v ? sti[e] : 0u);
+  }
+}
+
+}  // namespace airtopk
