@@ -505,6 +505,10 @@ def launch_names(plan):
         return ["batch_kernel (sample + window stream + finish)", "cluster_kernel (fallback rows)"], [True, False]
     P = plan["passes"]
     L = plan["launches"]
+    if plan["engine"] == 1 and L in (1, 3):  # fused tail: [sample, window pass,] one launch for the rest
+        if L == 1:
+            return ["tail_kernel (all passes, from L)"], [True]
+        return ["sample_kernel", "window_pass (DF=3)", "tail_kernel (remaining passes)"], [False, True, False]
     if L not in (P + 1, P + 3):  # window pass + tail_q grid passes + one cluster-engine tail launch
         tq = L - 3
         names = ["sample_kernel", "window_pass (DF=3)"] + [f"pass_kernel q={q} [window buffer]" for q in range(tq)]

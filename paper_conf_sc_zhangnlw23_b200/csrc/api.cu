@@ -131,7 +131,10 @@ Plan make_plan(const SelectArgs& a) {
   const size_t csz = isz;  // histogram counter width
   p.off_state = 0;
   p.off_hist = align_up(sizeof(RowState) * (size_t)a.batch, 256);
-  p.off_bcode = p.off_hist + align_up((size_t)a.batch * 2 * kMaxBins * csz, 256);
+  // fused tail (batch 1): 3 rotating histograms + per-pass buffer counts, zeroed with the state
+  p.off_thist = p.off_hist + align_up((size_t)a.batch * 2 * kMaxBins * csz, 256);
+  p.off_tcnt = p.off_thist + (a.batch == 1 ? align_up((size_t)3 * kMaxBins * csz, 256) : 0);
+  p.off_bcode = p.off_tcnt + (a.batch == 1 ? 256 : 0);
   p.off_bidx = p.off_bcode + align_up((size_t)2 * a.batch * p.cap_alloc * key_bytes(a.kind), 256);
   // sample-guided window (grid engine, position indices): stratified samples, 4K..16K
   p.nsamp = 0;
@@ -268,6 +271,10 @@ static void choose_launch(const SelectArgs& a, Plan& p) {
       p.csize = a.cluster_size > 0 ? a.cluster_size : cs;
     }
   }
+  // batch 1 (no trace, no tail): every pass after the window pass in one cooperative launch
+  // (window = -1 keeps the paper's one-kernel-per-pass structure: the P:146-156 ablations)
+  p.fused = (p.engine == 1 && a.batch == 1 && !a.in_idx && a.trace == nullptr && !p.tail && a.window >= 0 &&
+             getenv("AIRTOPK_NO_FUSED") == nullptr) ? 1 : 0;
   // bulk-copy streaming for a few long rows (every SM busy with 1 CTA); register loads otherwise
   p.tma = 0;
   if (!a.in_idx && !p.idx64 && a.tma >= 0 &&
@@ -577,6 +584,7 @@ airtopk_status airtopk_describe(airtopk_dtype dtype, int64_t batch, int64_t len,
   out->engine = p.engine;
   out->passes = p.P;
   out->launches = (p.engine == 3 || p.engine == 4 || p.engine == 6) ? 1 : (p.engine == 2 ? 1 : p.engine == 5 ? 2
+                  : p.fused ? 1 + (p.nsamp > 0 ? 2 : 0)
                   : (p.tail ? 3 + p.tail_q : p.P + 1 + (p.nsamp > 0 ? 2 : 0)));
   out->ctas_per_row = (p.engine == 1 || p.engine == 4) ? p.cpr : 0;
   out->cluster_size = (p.engine == 2 || p.engine == 5 || p.engine == 6 || p.tail) ? p.csize : 0;

@@ -119,6 +119,11 @@ struct alignas(128) RowState {
   unsigned long long win_nmin, win_max;  // ~min and max code of the window members (atomicMax)
 };
 
+// no-op debug-stamp callback (kernels take a Stamp functor for optional %globaltimer stamps)
+struct NoStamp {
+  __device__ void operator()(int) const {}
+};
+
 template <typename T>
 __device__ __forceinline__ T shfl(T v, int src) {
   if constexpr (sizeof(T) == 8) {

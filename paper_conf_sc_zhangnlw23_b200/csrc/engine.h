@@ -47,6 +47,7 @@ struct Plan {
   int tail;          // grid engine: finish after the window pass with one cluster-engine launch
   int tail_q;        // ... after the grid passes q < tail_q (0: right after the window pass)
   int tma;           // grid engine: stream rows through bulk-copy (TMA) shared rings, 1 CTA/SM
+  int fused;         // grid engine, batch 1: every pass after the window pass in one cooperative launch
   // batched engine (engine 5, engine_batch.cuh): eligible by shape; slot geometry
   int batch_ok;      // the shape qualifies (alignment is checked at run time)
   int bnsamp;        // samples per row
@@ -54,7 +55,8 @@ struct Plan {
   int nwc;           // (chunk, warp) slots per row
   int scap;          // entries per slot
   int rslice;        // resident-cluster engine: keys per CTA
-  size_t off_state, off_hist, off_bcode, off_bidx, off_samp, off_bcnt, off_bslot, off_bsidx, off_bfail, bytes;
+  size_t off_state, off_hist, off_thist, off_tcnt, off_bcode, off_bidx, off_samp, off_bcnt, off_bslot, off_bsidx,
+      off_bfail, bytes;
 };
 
 // cudaFuncSetAttribute once per (kernel, current device, attribute, value): the runtime applies

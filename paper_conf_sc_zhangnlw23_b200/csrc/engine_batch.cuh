@@ -66,7 +66,6 @@ static_assert(kBVT * 16 * kBGThreads == (int)kBStage, "stage = group threads x k
 static_assert(kBStages % kBGroups == 0, "a stage always belongs to the same group");
 static_assert(kBGWarps == kBatchSlotWarps, "host/device slot geometry");
 constexpr int kBFcap = kBatchFcap;            // entries (results + members) one row may stage in the finish
-constexpr int kBBrute = 1024;                 // sample-rank selection: brute-force rank below this many
 constexpr size_t kBRingBytes = (size_t)kBStages * kBStage;
 static_assert((size_t)kMaxSamples * 4 <= (size_t)(kBStages - kBPre) * kBStage, "samples fit the unused stages");
 
@@ -105,7 +104,7 @@ __device__ __forceinline__ void bstamp(const BatchParams& p, int f) {
 template <typename W>
 struct BatchShared {
   unsigned hist[kMaxBins];
-  W brute[kBBrute];             // compacted candidates of the rank selection
+  W brute[kRankBrute];          // compacted candidates of the rank selection
   unsigned long long tmp[kBWarps];
   ScanResult res;
   W wmin[kBWarps], wmax[kBWarps];
@@ -117,75 +116,6 @@ struct BatchShared {
 };
 
 // ---------------------------------------------------------------------------------- phase A
-// Sample order statistic of rank `rank` among the samples s[0..ns) (shared memory), all threads.
-// MSD digits of up to 11 bits below the bits on which every sample agrees (prefix); once at most
-// kBBrute samples share the prefix they are compacted and ranked by counting.
-template <typename W, typename Stamp = NoStamp>
-__device__ W sample_rank(const W* s, int ns, int rank, W smin, W smax, BatchShared<W>& sh, Stamp stamp = Stamp()) {
-  constexpr int WB = 8 * (int)sizeof(W);
-  const W diff = smin ^ smax;
-  int hb = diff ? (WB - (sizeof(W) == 8 ? __clzll((long long)diff) : __clz((int)diff))) : 0;
-  W mask = (hb >= WB) ? (W)0 : (W)(~(W)0 << hb);
-  W prefix = smin & mask;
-  int cnt = ns;
-  while (true) {
-    if (hb == 0) return prefix;
-    if (cnt <= kBBrute) {
-      if (threadIdx.x == 0) sh.cnt = 0;
-      __syncthreads();
-#pragma unroll 1
-      for (int i = threadIdx.x; i < ns; i += kBBlock) {
-        const W x = s[i];
-        const bool m = (x & mask) == prefix;
-        const unsigned b = __ballot_sync(kFull, m);
-        unsigned base = 0;
-        if ((threadIdx.x & 31) == 0 && b) base = atomicAdd(&sh.cnt, (unsigned)__popc(b));
-        base = __shfl_sync(kFull, base, 0);
-        if (m) sh.brute[base + __popc(b & lanemask_lt())] = x;
-      }
-      __syncthreads();
-      stamp(3);
-      if ((int)threadIdx.x < cnt) {
-        const W x = sh.brute[threadIdx.x];
-        int less = 0, eq = 0;
-#pragma unroll 4
-        for (int j = 0; j < cnt; ++j) {
-          const W y = sh.brute[j];
-          less += y < x;
-          eq += y == x;
-        }
-        if (less <= rank && rank < less + eq) sh.result = x;
-      }
-      __syncthreads();
-      stamp(4);
-      const W r = sh.result;
-      __syncthreads();
-      return r;
-    }
-    const int shf = hb > kDigitBits ? hb - kDigitBits : 0, w = hb - shf;
-    const unsigned dm = (1u << w) - 1u;
-    for (int i = threadIdx.x; i < (1 << w); i += kBBlock) sh.hist[i] = 0;
-    __syncthreads();
-    stamp(0);
-#pragma unroll 1
-    for (int i = threadIdx.x; i < ns; i += kBBlock) {
-      const W x = s[i];
-      if ((x & mask) == prefix) atomicAdd(&sh.hist[(unsigned)(x >> shf) & dm], 1u);
-    }
-    __syncthreads();
-    stamp(1);
-    const ScanResult r = scan_choose<kBBlock>([&](int b) { return (unsigned long long)sh.hist[b]; }, 1 << w,
-                                             (unsigned long long)rank + 1, sh.tmp, &sh.res);
-    stamp(2);
-    rank -= (int)r.before;
-    cnt = (int)r.cnt;
-    prefix |= (W)r.j << shf;
-    mask |= (W)dm << shf;
-    hb = shf;
-  }
-}
-
-// Phase A for one row (all threads): window [lo, hi] from the sample order statistics.
 template <typename U>
 __device__ __forceinline__ void batch_issue(const BatchParams& p, int64_t ch, unsigned ring, int stage);
 template <typename U>
@@ -264,8 +194,8 @@ __device__ void batch_sample_row(const BatchParams& p, int64_t row, void* samp_v
   if (rhi >= ns - 1) {
     state = 3;
   } else {
-    hi = sample_rank<W>(s, ns, rhi, smin, smax, sh, [&](int f) { bstamp(p, 16 + f); });
-    lo = rlo > 0 ? sample_rank<W>(s, ns, rlo, smin, smax, sh) : (W)0;  // none below the window if rlo <= 0
+    hi = sample_rank<W, kBBlock>(s, ns, rhi, smin, smax, sh, [&](int f) { bstamp(p, 16 + f); });
+    lo = rlo > 0 ? sample_rank<W, kBBlock>(s, ns, rlo, smin, smax, sh) : (W)0;  // none below the window if rlo <= 0
     bstamp(p, 2);
     // estimated entries (results + members: every code <= hi) vs the finish capacity
     unsigned le = 0;

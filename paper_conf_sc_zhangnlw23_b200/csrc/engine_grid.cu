@@ -77,6 +77,8 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t
   gp.nsms = num_sms();
   gp.early_stop = a.early_stop;
   gp.idx_off = a.idx_off;
+  gp.thist = base + pl.off_thist;
+  gp.tcnt = (unsigned long long*)(base + pl.off_tcnt);
   {
     static const char* env2 = getenv("AIRTOPK_SMALL_FINISH");  // A/B knob (0 = off)
     gp.small_finish = env2 ? std::min(atoi(env2), kSmallFinish) : kSmallFinish;

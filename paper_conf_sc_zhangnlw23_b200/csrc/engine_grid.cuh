@@ -39,10 +39,14 @@
 #pragma once
 
 #include <algorithm>
+#include <cstdlib>
 #include <type_traits>
+
+#include <cooperative_groups.h>
 
 #include "device.cuh"
 #include "engine.h"
+#include "finish.cuh"
 #include "passes.cuh"
 
 namespace airtopk {
@@ -68,6 +72,8 @@ struct GridParams {
   int small_finish;  // a buffer-source pass over <= this many entries finishes the row in one CTA
   int early_stop;   // 0 on, -1 off (ablation)
   int64_t idx_off;  // added to every output index (airtopk_select_shard)
+  void* thist;      // fused tail (batch 1): 3 rotating global histograms
+  unsigned long long* tcnt;  // fused tail: candidates stored by pass q (zeroed with the state)
 };
 
 constexpr int kBlock = 512;
@@ -379,10 +385,6 @@ constexpr int kBrute = 128;
 constexpr int kSampleHistCopies = 4;
 static_assert(kSampleBlock / 8 >= kBrute, "8 threads per bin member in the brute-force rank");
 
-struct NoStamp {
-  __device__ void operator()(int) const {}
-};
-
 template <typename W, int PER, typename Stamp = NoStamp>
 __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo, int rhi, W pmin, int hb,
                                  unsigned* hist /* 2048 x copies */, unsigned* wsum /* 32 */, W* shw, int* cnt,
@@ -524,6 +526,20 @@ __device__ void block_select_two(const W (&v)[PER], int tv, W* scratch, int rlo,
   hi = res[1];
 }
 
+#ifndef AIRTOPK_SAMPLE_LEAN
+#define AIRTOPK_SAMPLE_LEAN 1
+#endif
+// shared scratch of sample_rank (aliases the sample kernel's histogram array)
+template <typename W>
+struct SampleRankShared {
+  unsigned hist[kMaxBins];
+  W brute[kRankBrute];
+  unsigned long long tmp[32];
+  ScanResult res;
+  W result;
+  unsigned cnt;
+};
+
 constexpr int kSampleCTAs = 16;  // max CTAs per row issuing the scattered sample loads (one SM cannot
                                  // keep 16K independent DRAM loads in flight)
 
@@ -535,7 +551,7 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
   extern __shared__ __align__(16) unsigned char sample_smem[];
   W* scratch = (W*)sample_smem;  // nsamp entries: compacted bins of the rank selection (last CTA)
-  __shared__ unsigned hist[2048 * kSampleHistCopies];
+  __shared__ __align__(16) unsigned hist[2048 * kSampleHistCopies];
   __shared__ unsigned wsum[32];
   __shared__ W shw[8];
   __shared__ int sh_cnt[4];
@@ -652,8 +668,21 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
   stamp(5);
   // no results below the window when rlo <= 0: everything up to hi is a candidate
   W lo, hi;
+#if AIRTOPK_SAMPLE_LEAN
+  // the samples into shared memory, then the lean rank selection (finish.cuh: MSD digit histograms,
+  // counting rank once <= 1024 samples share the prefix; measured ~2x faster than the register
+  // version below, whose unrolled code runs once per select on a cold instruction cache)
+  (void)hb;
+#pragma unroll
+  for (int t = 0; t < PER; ++t)
+    if (t < tv) scratch[t * kSampleBlock + threadIdx.x] = v[t];
+  __syncthreads();
+  hi = sample_rank<W, kSampleBlock>(scratch, nsamp, rhi, smin, smax, *(SampleRankShared<W>*)hist);
+  lo = rlo > 0 ? sample_rank<W, kSampleBlock>(scratch, nsamp, rlo, smin, smax, *(SampleRankShared<W>*)hist) : (W)0;
+#else
   block_select_two<W, PER>(v, tv, scratch, rlo <= 0 ? -1 : rlo, rhi, smin, hb, hist, wsum, shw, sh_cnt, lo, hi);
   if (rlo <= 0) lo = 0;
+#endif
   stamp(6);
   // Estimated window size from the sample (ties at hi included): a window that would overflow the
   // candidate buffer (e.g. a row of equal keys) is not tried — the paper's passes run instead.
@@ -789,6 +818,204 @@ cudaError_t launch_grid_passes(const GridParams& gp, int64_t batch, int nsamp, c
   return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------------------------------------
+// Fused tail (batch 1): every pass after the window pass — or, when the window missed or there was
+// none, every pass of the paper from L — in ONE cooperative launch. The per-pass kernel boundary of
+// Algorithm 1 and its last-CTA scan become a grid-wide barrier after which EVERY
+// CTA scans the merged histogram itself (identical j, K, C everywhere; no second barrier), so a
+// pass over a small candidate buffer costs a barrier instead of a launch (measured: the passes
+// after the c4 window pass took ~58 us as 6 launches). Histograms rotate over 3 global slots (slot
+// (q+2) % 3 is zeroed during pass q: every CTA finished scanning it before the barrier of pass q);
+// the buffer counts are per pass (zeroed with the row state).
+struct TailState {
+  unsigned long long K, C, tcode, tidx, nbuf;
+  int src1;   // 0 = input row L, s + 1 = candidate buffer slot s
+  int stop1;  // 1 + digit after whose scan K == C (early stop); 0 = none
+};
+
+template <int KIND, typename IdxT, int DF, int DH>
+__device__ __forceinline__ bool tail_pass(const GridParams& p, int q, TailState& S, unsigned* sh_hist,
+                                          WarpQ<typename KT<KIND>::U, IdxT>* wq, unsigned long long* sh_tmp,
+                                          ScanResult* sh_res) {
+  namespace cg = cooperative_groups;
+  using U = typename KT<KIND>::U;
+  using CountT = std::conditional_t<sizeof(IdxT) == 8, unsigned long long, unsigned>;
+  constexpr bool FILTER = (DF == 1 || DF == 2);
+  const int tid = threadIdx.x;
+  RowState* st = p.st;
+  PassCtx<U, IdxT> c;
+  c.q = q;
+  c.emit_all = FILTER && ((S.stop1 != 0 && S.stop1 - 1 == q - 1) || DH == 0);
+  c.do_hist = (DH != 0) && !c.emit_all;
+  const unsigned long long Cin = FILTER ? S.C : (unsigned long long)p.len;
+  c.srcL = (S.src1 == 0);
+  c.store = c.do_hist && FILTER && (Cin <= (unsigned long long)p.cap_rule);  // Alg1 L17
+  c.sel_min = p.sel_min != 0;
+  c.reverse = (q & 1) != 0;
+  c.dh = digit_of(q, KT<KIND>::R, p.IB);
+  c.dh2 = c.dh;
+  c.df = digit_of(FILTER ? q - 1 : 0, KT<KIND>::R, p.IB);
+  c.tcode = S.tcode;
+  c.tidx = S.tidx;
+  c.wnmin = nullptr;
+  c.wmax = nullptr;
+  c.lo = 0;
+  c.span1 = 0;
+  c.rowp = (const U*)p.keys;
+  c.rowi = nullptr;
+  c.len = p.len;
+  c.slice = blockIdx.x;
+  c.nslices = gridDim.x;
+  const int islot = S.src1 > 0 ? S.src1 - 1 : 0;
+  const int sslot = (S.src1 == 1) ? 1 : 0;  // the buffer this pass writes
+  c.bcin = (const U*)p.bcode + (size_t)islot * p.cap_alloc;
+  c.biin = (const IdxT*)p.bidx + (size_t)islot * p.cap_alloc;
+  c.nbuf = S.src1 > 0 ? S.nbuf : 0ull;
+  c.ov = (U*)p.out_vals;
+  c.oi = p.out_idx;
+  c.ioff = p.idx_off;
+  c.outc = &st->out_count;
+  c.kk = (unsigned long long)p.k;
+  c.bco = (U*)p.bcode + (size_t)sslot * p.cap_alloc;
+  c.bio = (IdxT*)p.bidx + (size_t)sslot * p.cap_alloc;
+  c.bufc = p.tcnt + q;
+  c.capa = (unsigned long long)p.cap_alloc;
+  c.err = &st->error;
+  c.hist = sh_hist;
+  c.ring = 0;
+  c.wq = &wq[tid >> 5];
+  if constexpr (FILTER && DH != 0) {
+    // small finish: one CTA ends the row; the decision is grid-uniform
+    if (!c.emit_all && !c.srcL && c.nbuf <= (unsigned long long)p.small_finish) {
+      if (blockIdx.x == 0)
+        small_finish<KIND, IdxT, kBlock>(c, S.K, (U*)sh_hist, (IdxT*)((unsigned char*)sh_hist + kSmallFinish * sizeof(U)));
+      return true;
+    }
+  }
+  constexpr int HC = hist_copies<KIND, IdxT, DF>();
+  if (c.do_hist || DF == 0) {
+    for (int i = tid; i < kHistSlots * HC; i += kBlock) sh_hist[i] = 0;
+    __syncthreads();
+  }
+  run_pass<KIND, IdxT, DF, DH, false, kBlock, 0, false, kGridBU>(c);
+  if (!(c.do_hist || DF == 0)) return true;  // emit-all pass: the row is complete
+  __syncthreads();
+  CountT* gh = (CountT*)p.thist + (size_t)(q % 3) * kMaxBins;
+  const int nb = 1 << c.dh.width;
+  for (int i = tid; i < nb; i += kBlock) {
+    unsigned v = 0;
+#pragma unroll
+    for (int h = 0; h < HC; ++h) v += sh_hist[i * HC + h];
+    if (v) atomicAdd(&gh[i], (CountT)v);
+  }
+  cg::this_grid().sync();  // every CTA's histogram, results and candidates of pass q are published
+  const ScanResult r = scan_choose<kBlock>([&](int b) { return (unsigned long long)__ldcg(&gh[b]); }, nb, S.K, sh_tmp,
+                                           sh_res);
+  if (blockIdx.x == 0) {
+    CountT* gz = (CountT*)p.thist + (size_t)((q + 2) % 3) * kMaxBins;
+    for (int i = tid; i < kMaxBins; i += kBlock) gz[i] = 0;
+  }
+  const unsigned long long newK = S.K - r.before, newC = r.cnt;  // Alg1 L26-28
+  if (c.store) {
+    S.src1 = sslot + 1;
+    S.nbuf = __ldcg(c.bufc);
+  }
+  S.C = newC;
+  S.K = newK;
+  if (!c.dh.is_idx) S.tcode |= (unsigned long long)r.j << c.dh.shift;
+  else S.tidx |= (unsigned long long)r.j << c.dh.shift;
+  if (newK == newC && p.early_stop == 0) S.stop1 = q + 1;  // early stop
+  if (blockIdx.x == 0 && tid == 0) {
+    st->K = newK;
+    st->C = newC;
+    st->Cp = Cin;
+    st->tcode = S.tcode;
+    st->tidx = S.tidx;
+    st->j = r.j;
+    st->npass = q + 1;
+    st->stop1 = S.stop1;
+    st->src1 = S.src1;
+    if (r.total != Cin) st->error |= 4u;
+  }
+  return false;
+}
+
+template <int KIND, typename IdxT>
+__global__ void __launch_bounds__(kBlock, kMinBlocksFilter) tail_kernel(const GridParams p) {
+  using U = typename KT<KIND>::U;
+  extern __shared__ unsigned sh_hist[];
+  __shared__ WarpQ<U, IdxT> sh_wq[kWarps];
+  __shared__ unsigned long long sh_tmp[kWarps];
+  __shared__ ScanResult sh_res;
+  pdl_wait();  // the window pass (previous launch) is complete
+  const RowState* st = p.st;
+  TailState S;
+  int q;
+  if (st->win_state == 1) {  // continue after the window pass (its scan fixed digits < npass)
+    q = st->npass;
+    S.K = st->K;
+    S.C = st->C;
+    S.tcode = st->tcode;
+    S.tidx = st->tidx;
+    S.src1 = st->src1;
+    S.stop1 = st->stop1;
+    S.nbuf = S.src1 > 0 ? st->buf_count[S.src1 - 1] : 0ull;
+  } else {  // no window / the window missed: the paper's passes from L
+    q = 0;
+    S.K = (unsigned long long)p.k;
+    S.C = (unsigned long long)p.len;
+    S.tcode = S.tidx = 0;
+    S.src1 = 0;
+    S.stop1 = 0;
+    S.nbuf = 0;
+  }
+#pragma unroll 1
+  for (; q <= p.P; ++q) {
+    if (S.stop1 != 0 && S.stop1 - 1 < q - 1) break;
+    const int DF = q == 0 ? 0 : (digit_of(q - 1, KT<KIND>::R, p.IB).is_idx ? 2 : 1);
+    const int DH = q == p.P ? 0 : (digit_of(q, KT<KIND>::R, p.IB).is_idx ? 2 : 1);
+    bool done;
+    switch (DF * 3 + DH) {
+      case 0 * 3 + 1: done = tail_pass<KIND, IdxT, 0, 1>(p, q, S, sh_hist, sh_wq, sh_tmp, &sh_res); break;
+      case 1 * 3 + 1: done = tail_pass<KIND, IdxT, 1, 1>(p, q, S, sh_hist, sh_wq, sh_tmp, &sh_res); break;
+      case 1 * 3 + 2: done = tail_pass<KIND, IdxT, 1, 2>(p, q, S, sh_hist, sh_wq, sh_tmp, &sh_res); break;
+      case 2 * 3 + 2: done = tail_pass<KIND, IdxT, 2, 2>(p, q, S, sh_hist, sh_wq, sh_tmp, &sh_res); break;
+      default: done = tail_pass<KIND, IdxT, 2, 0>(p, q, S, sh_hist, sh_wq, sh_tmp, &sh_res); break;
+    }
+    if (done) break;
+  }
+}
+
+template <int KIND, typename IdxT>
+cudaError_t launch_tail(const GridParams& gp, cudaStream_t s) {
+  auto kern = tail_kernel<KIND, IdxT>;
+  constexpr size_t smem = (size_t)kHistSlots * 4 * kHistCopies;
+  static_assert((size_t)kHistSlots * 4 * kHistCopies >= (size_t)kSmallFinish * (sizeof(typename KT<KIND>::U) + sizeof(IdxT)),
+                "small finish smem");
+  cudaError_t e = func_attr(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  if (!occ_cache_get((const void*)kern, 0, &occ)) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, smem);
+    if (e != cudaSuccess) return e;
+    occ_cache_put((const void*)kern, 0, occ);
+  }
+  if (occ < 1) return cudaErrorInvalidConfiguration;
+  cudaLaunchConfig_t cfg = {};
+  int G = gp.nsms * std::min(occ, kMinBlocksFilter);
+  if (const char* env = getenv("AIRTOPK_TAIL_CTAS")) G = std::min(G, std::max(1, atoi(env)));  // A/B knob
+  cfg.gridDim = dim3((unsigned)G);
+  cfg.blockDim = dim3(kBlock);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, gp);
+}
+
 template <int KIND>
 cudaError_t launch_cluster_kind(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t s, int tail);
 
@@ -799,6 +1026,15 @@ cudaError_t launch_grid_kind(const SelectArgs& a, const Plan& pl, const GridPara
   const Events ev{a.events, a.n_events};
   if (a.in_idx) return launch_grid_passes<KIND, uint64_t, true>(gp, a.batch, 0, ev, s);
   cudaError_t e;
+  if (pl.fused) {  // sample + window pass, then ONE cooperative launch for every remaining pass
+    e = pl.idx64 ? launch_grid_passes<KIND, uint64_t, false>(gp, a.batch, pl.nsamp, ev, s, 0)
+        : pl.tma ? launch_grid_passes<KIND, uint32_t, false, true>(gp, a.batch, pl.nsamp, ev, s, 0)
+                 : launch_grid_passes<KIND, uint32_t, false>(gp, a.batch, pl.nsamp, ev, s, 0);
+    if (e != cudaSuccess) return e;
+    e = pl.idx64 ? launch_tail<KIND, uint64_t>(gp, s) : launch_tail<KIND, uint32_t>(gp, s);
+    ev.record(pl.nsamp > 0 ? 3 : 1, s);
+    return e;
+  }
   const int upto = pl.tail ? pl.tail_q : (1 << 30);
   if (pl.idx64) e = launch_grid_passes<KIND, uint64_t, false>(gp, a.batch, pl.nsamp, ev, s, upto);
   else if (pl.tma) e = launch_grid_passes<KIND, uint32_t, false, true>(gp, a.batch, pl.nsamp, ev, s, upto);

@@ -125,4 +125,79 @@ __device__ void block_select_smem(const typename KT<KIND>::U* stc, const unsigne
   }
 }
 
+// Sample order statistic of rank `rank` among s[0..ns) (shared memory), all BLOCK threads: MSD
+// digits of up to 11 bits below the bits on which every sample agrees; once at most kRankBrute
+// samples share the prefix they are compacted and ranked by counting. SH provides hist[kMaxBins],
+// brute[kRankBrute], tmp[BLOCK / 32], res, result, cnt (shared memory).
+constexpr int kRankBrute = 1024;
+
+// Sample order statistic of rank `rank` among the samples s[0..ns) (shared memory), all threads.
+// MSD digits of up to 11 bits below the bits on which every sample agrees (prefix); once at most
+// kRankBrute samples share the prefix they are compacted and ranked by counting.
+template <typename W, int BLOCK, typename SH, typename Stamp = NoStamp>
+__device__ W sample_rank(const W* s, int ns, int rank, W smin, W smax, SH& sh, Stamp stamp = Stamp()) {
+  constexpr int WB = 8 * (int)sizeof(W);
+  const W diff = smin ^ smax;
+  int hb = diff ? (WB - (sizeof(W) == 8 ? __clzll((long long)diff) : __clz((int)diff))) : 0;
+  W mask = (hb >= WB) ? (W)0 : (W)(~(W)0 << hb);
+  W prefix = smin & mask;
+  int cnt = ns;
+  while (true) {
+    if (hb == 0) return prefix;
+    if (cnt <= kRankBrute) {
+      if (threadIdx.x == 0) sh.cnt = 0;
+      __syncthreads();
+#pragma unroll 1
+      for (int i = threadIdx.x; i < ns; i += BLOCK) {
+        const W x = s[i];
+        const bool m = (x & mask) == prefix;
+        const unsigned b = __ballot_sync(kFull, m);
+        unsigned base = 0;
+        if ((threadIdx.x & 31) == 0 && b) base = atomicAdd(&sh.cnt, (unsigned)__popc(b));
+        base = __shfl_sync(kFull, base, 0);
+        if (m) sh.brute[base + __popc(b & lanemask_lt())] = x;
+      }
+      __syncthreads();
+      stamp(3);
+      if ((int)threadIdx.x < cnt) {
+        const W x = sh.brute[threadIdx.x];
+        int less = 0, eq = 0;
+#pragma unroll 4
+        for (int j = 0; j < cnt; ++j) {
+          const W y = sh.brute[j];
+          less += y < x;
+          eq += y == x;
+        }
+        if (less <= rank && rank < less + eq) sh.result = x;
+      }
+      __syncthreads();
+      stamp(4);
+      const W r = sh.result;
+      __syncthreads();
+      return r;
+    }
+    const int shf = hb > kDigitBits ? hb - kDigitBits : 0, w = hb - shf;
+    const unsigned dm = (1u << w) - 1u;
+    for (int i = threadIdx.x; i < (1 << w); i += BLOCK) sh.hist[i] = 0;
+    __syncthreads();
+    stamp(0);
+#pragma unroll 1
+    for (int i = threadIdx.x; i < ns; i += BLOCK) {
+      const W x = s[i];
+      if ((x & mask) == prefix) atomicAdd(&sh.hist[(unsigned)(x >> shf) & dm], 1u);
+    }
+    __syncthreads();
+    stamp(1);
+    const ScanResult r = scan_choose<BLOCK>([&](int b) { return (unsigned long long)sh.hist[b]; }, 1 << w,
+                                             (unsigned long long)rank + 1, sh.tmp, &sh.res);
+    stamp(2);
+    rank -= (int)r.before;
+    cnt = (int)r.cnt;
+    prefix |= (W)r.j << shf;
+    mask |= (W)dm << shf;
+    hb = shf;
+  }
+}
+
+// Phase A for one row (all threads): window [lo, hi] from the sample order statistics.
 }  // namespace airtopk
