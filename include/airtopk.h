@@ -89,12 +89,21 @@ typedef enum {
   AIRTOPK_ENGINE_AUTO = 0,
   AIRTOPK_ENGINE_GRID = 1,    /* multi-CTA per row, one launch per pass, last-CTA scan */
   AIRTOPK_ENGINE_CLUSTER = 2, /* one thread-block cluster per row, all passes in one launch */
-  AIRTOPK_ENGINE_GRIDSELECT = 4 /* the paper's second algorithm (§4): per-warp shared
+  AIRTOPK_ENGINE_GRIDSELECT = 4, /* the paper's second algorithm (§4): per-warp shared
                                    32-entry queue with two-step ballot insertion, sorted per-warp
-                                   top-K lists merged by the last CTA of the row. Same results
-                                   (lowest-index ties). Only for keys of <= 32 bits, len < 2^32 and
-                                   K <= 256, else AIRTOPK_EINVAL. Rows come out sorted. Never chosen
-                                   by AUTO. */
+                                   top-K lists, a row-wide shared threshold, CTA lists merged by the
+                                   last CTA of the row. Same results (lowest-index ties). Only for
+                                   keys of <= 32 bits, len < 2^32 and K <= 2048, else
+                                   AIRTOPK_EINVAL. Rows come out sorted. Never chosen by AUTO. */
+  AIRTOPK_ENGINE_BATCH = 5,     /* batched rows in ONE cooperative launch: per-row sample window,
+                                   single read of every row into fixed per-(chunk, warp) slots,
+                                   per-row shared-memory finish; rows whose window fails are redone
+                                   by a cluster-engine launch. Needs 16-byte aligned rows and a
+                                   window that fits 16K entries per row, else AIRTOPK_EINVAL. */
+  AIRTOPK_ENGINE_RESIDENT = 6,  /* rows of <= 512K keys (256K for f64) held in the shared memory of
+                                   a thread-block cluster: one HBM read, every pass on chip. */
+  AIRTOPK_ENGINE_GRIDSELECT_PTQ = 7 /* GridSelect with per-thread register queues instead of the
+                                   shared queue: the Fig. 11 ablation. Same scope. */
 } airtopk_engine;
 
 /* Tuning / ablation knobs. Pass NULL for the defaults. */
@@ -104,7 +113,7 @@ typedef struct {
                            whenever at least one element was eliminated. Must be >= 0. */
   int32_t engine;       /* airtopk_engine; 0 = auto */
   int32_t ctas_per_row; /* grid engine: CTAs per row; 0 = auto (fills the 148 SMs) */
-  int32_t cluster_size; /* cluster engine: CTAs per cluster (1,2,4,8,16); 0 = auto */
+  int32_t cluster_size; /* cluster / resident engine: CTAs per cluster (1,2,4,8,16); 0 = auto */
   int32_t n_events;     /* number of entries in `events` */
   int64_t* trace;       /* optional DEVICE buffer of batch * AIRTOPK_TRACE_MAX_PASSES * 10 int64:
                            per-row state after each scan (width, src_is_input, stored, j, K, C, C',

@@ -12,11 +12,11 @@ import ctypes
 
 from . import _lib
 from ._lib import (AirTopKError, Options, OK, ENGINE_AUTO, ENGINE_GRID, ENGINE_CLUSTER, ENGINE_GRIDSELECT,
-                   ENGINE_BATCH, TRACE_MAX_PASSES)
+                   ENGINE_BATCH, ENGINE_RESIDENT, ENGINE_GRIDSELECT_PTQ, TRACE_MAX_PASSES)
 
 __all__ = ["select", "select_with_idx", "select_shard", "merge_idx_bits", "select_host", "workspace_bytes",
            "describe", "lib", "AirTopKError", "DeviceError", "ENGINE_AUTO", "ENGINE_GRID", "ENGINE_CLUSTER",
-           "ENGINE_GRIDSELECT", "ENGINE_BATCH", "dtype_code"]
+           "ENGINE_GRIDSELECT", "ENGINE_BATCH", "ENGINE_RESIDENT", "ENGINE_GRIDSELECT_PTQ", "dtype_code"]
 
 _LIB = None
 

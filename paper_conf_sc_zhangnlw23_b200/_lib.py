@@ -13,7 +13,8 @@ LIB_PATH = os.environ.get("AIRTOPK_LIB", os.path.join(_PKG, "libairtopk.so"))
 OK, EINVAL, EDTYPE, ENOSPACE, ECUDA, EDEVICE = 0, 1, 2, 3, 4, 5
 ERR_OUTPUT_OVERFLOW, ERR_BUFFER_OVERFLOW, ERR_COUNT = 1, 2, 4
 F32, F16, BF16, F64, U32 = 0, 1, 2, 3, 4
-ENGINE_AUTO, ENGINE_GRID, ENGINE_CLUSTER, ENGINE_GRIDSELECT, ENGINE_BATCH = 0, 1, 2, 4, 5
+ENGINE_AUTO, ENGINE_GRID, ENGINE_CLUSTER, ENGINE_GRIDSELECT, ENGINE_BATCH, ENGINE_RESIDENT, ENGINE_GRIDSELECT_PTQ = \
+    0, 1, 2, 4, 5, 6, 7
 TRACE_MAX_PASSES = 16
 TRACE_FIELDS = ("width", "src_L", "stored", "j", "K", "C", "Cp", "emitted", "early_stop", "read")
 

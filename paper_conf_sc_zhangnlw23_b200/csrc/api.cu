@@ -113,7 +113,7 @@ Plan make_plan(const SelectArgs& a) {
     p.engine = 3;
     return p;
   }
-  if (a.engine == 4) {  // GridSelect (the paper's second algorithm)
+  if (a.engine == 4 || a.engine == 7) {  // GridSelect (the paper's second algorithm; 7: per-thread queues)
     p.engine = 4;
     p.cpr = gridselect_ctas(a);
     p.bytes = gridselect_workspace(a, p.cpr);
@@ -225,7 +225,7 @@ static void resident_geometry(const SelectArgs& a, Plan& p) {
 }
 
 static void choose_launch(const SelectArgs& a, Plan& p) {
-  if (p.engine == 3 || p.engine == 4) return;
+  if (p.engine == 3 || p.engine == 4) return;  // (4: GridSelect, either queue variant)
   // AUTO (tools/engine_ab.py, profiles/r02_engine_ab.txt, L2 flushed between selects): the
   // resident cluster wins for rows of <= 2^14 keys at any batch and for a single row of <= 2^16
   if (a.engine == 6 || (a.engine == 0 && a.window == 0 && resident_fits(a) && a.trace == nullptr &&
@@ -308,8 +308,8 @@ static airtopk_status validate(const SelectArgs& a) {
   if (!a.keys || !a.out_vals || !a.out_idx) return AIRTOPK_EINVAL;
   if (a.batch < 1 || a.len < 1 || a.k < 1 || a.k > a.len) return AIRTOPK_EINVAL;
   if (a.alpha < 0) return AIRTOPK_EINVAL;
-  if (a.engine < 0 || a.engine > 6 || a.engine == 3) return AIRTOPK_EINVAL;
-  if (a.engine == 4 && !gridselect_supported(a)) return AIRTOPK_EINVAL;
+  if (a.engine < 0 || a.engine > 7 || a.engine == 3) return AIRTOPK_EINVAL;
+  if ((a.engine == 4 || a.engine == 7) && !gridselect_supported(a)) return AIRTOPK_EINVAL;
   if (a.window < -1 || a.window > 1) return AIRTOPK_EINVAL;
   if (a.early_stop < -1 || a.early_stop > 0) return AIRTOPK_EINVAL;
   if (a.in_idx && (a.batch != 1 || a.idx_bits < 1 || a.idx_bits > 63)) return AIRTOPK_EINVAL;

@@ -80,8 +80,8 @@ def test_product_package_does_not_import_oracle():
 
 
 def test_gridselect_scope_validation_without_gpu():
-    """GridSelect (engine 4) accepts keys of <= 32 bits, len < 2^32, K <= 256 and
-    rejects the rest with AIRTOPK_EINVAL before touching the device."""
+    """GridSelect (engines 4 and 7) accepts keys of <= 32 bits, len < 2^32, K <= 2048
+     and rejects the rest with AIRTOPK_EINVAL before touching the device."""
     lib = at.lib()
     p = ctypes.c_void_p(256)
 
@@ -92,7 +92,10 @@ def test_gridselect_scope_validation_without_gpu():
 
     assert lib.airtopk_workspace_bytes_ex(0, 1, 1 << 16, 32, opts(4)) > 0        # f32, K = 32
     assert lib.airtopk_workspace_bytes_ex(1, 3, 1000, 256, opts(4)) > 0          # f16, K = 256
-    assert lib.airtopk_workspace_bytes_ex(0, 1, 1 << 16, 257, opts(4)) == 0      # K > 256
+    assert lib.airtopk_workspace_bytes_ex(0, 1, 1 << 16, 2048, opts(4)) > 0      # K = 2048
+    assert lib.airtopk_workspace_bytes_ex(0, 1, 1 << 16, 2048, opts(7)) > 0      # per-thread queues
+    assert lib.airtopk_workspace_bytes_ex(0, 1, 1 << 16, 2049, opts(4)) == 0     # K > 2048
+    assert lib.airtopk_workspace_bytes_ex(0, 1, 1 << 16, 32, opts(8)) == 0       # no engine 8
     assert lib.airtopk_workspace_bytes_ex(3, 1, 1 << 16, 32, opts(4)) == 0       # f64 keys
     assert lib.airtopk_workspace_bytes_ex(0, 1, 1 << 16, 32, opts(3)) == 0       # no engine 3
     assert lib.airtopk_select_ex(p, 3, 1, 100, 10, 1, p, p, p, 1 << 30, None, opts(4)) == _lib.EINVAL

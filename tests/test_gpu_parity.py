@@ -395,19 +395,30 @@ def test_row_longer_than_2p32(dtn, largest):
 
 @pytest.mark.parametrize("dist,m", [("uniform", 20), ("normal", 20), ("adversarial", 20), ("adversarial", 28)])
 @pytest.mark.parametrize("batch,n,k", [(1, 1 << 16, 32), (1, 1 << 16, 1), (3, 100003, 256), (5, 1000, 100),
-                                       (2, 33, 33), (4, 31, 7), (1, 1 << 20, 200)])
+                                       (2, 33, 33), (4, 31, 7), (1, 1 << 20, 200), (1, 1 << 20, 2048),
+                                       (2, 300001, 1500), (3, 5000, 1024)])
 @pytest.mark.parametrize("select_min", [True, False])
-def test_gridselect(dist, m, batch, n, k, select_min):
+@pytest.mark.parametrize("engine", [4, 7])
+def test_gridselect(dist, m, batch, n, k, select_min, engine):
+    """GridSelect with the shared queue (engine 4) and the per-thread-queue variant (engine 7, the
+    Fig. 11 ablation), K up to the paper's 2048."""
     x = _keys(dist, 131, batch, n, m=m)
-    v, i = gpu_select(x, "f32", k, select_min, engine=4)
+    v, i = gpu_select(x, "f32", k, select_min, engine=engine)
     assert_parity(x, "f32", k, select_min, v, i)
+
+
+def test_gridselect_rejects_k_above_2048():
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    with pytest.raises(at.AirTopKError):
+        at.select(torch.zeros((1, 5000), device="cuda"), 2049, engine=4)
 
 
 @pytest.mark.parametrize("dtn", ["f16", "bf16", "u32"])
 def test_gridselect_dtypes(dtn):
     u = gen.u64(92, 6 * 20011)
     raw = u.astype({"f16": np.uint16, "bf16": np.uint16, "u32": np.uint32}[dtn]).reshape(6, 20011)
-    for k in (1, 64, 256):
+    for k in (1, 64, 256, 2048):
         for sm in (True, False):
             v, i = gpu_select(raw, dtn, k, sm, engine=4)
             assert_parity(raw, dtn, k, sm, v, i)
