@@ -114,6 +114,47 @@ __device__ __noinline__ unsigned long long gs_flush(GsWarpView& w, int& cur, int
   return w.list[cur][K - 1];
 }
 
+// Merge two sorted lists A, B of K unique keys into out (the K smallest of the union), one warp:
+// A[i] lands at i + #{B < A[i]}, B[j] at j + #{A < B[j]} (binary searches; positions >= K dropped).
+__device__ __noinline__ void gs_merge2(const unsigned long long* A, const unsigned long long* B, unsigned long long* out,
+                                      int K) {
+  const int lane = threadIdx.x & 31;
+  for (int i = lane; i < K; i += 32) {
+    const unsigned long long a = A[i], b = B[i];
+    int lo = 0, hi = K;  // #{B < a}
+    while (lo < hi) {
+      const int mid = (lo + hi) >> 1;
+      if (B[mid] < a) lo = mid + 1; else hi = mid;
+    }
+    if (i + lo < K) out[i + lo] = a;
+    lo = 0;
+    hi = K;  // #{A < b}
+    while (lo < hi) {
+      const int mid = (lo + hi) >> 1;
+      if (A[mid] < b) lo = mid + 1; else hi = mid;
+    }
+    if (i + lo < K) out[i + lo] = b;
+  }
+  __syncwarp();
+}
+
+// The CTA's W sorted lists (buffer 0 of every warp) -> one, by a tree of pairwise merges (log2 W
+// levels, the merges of a level in parallel); returns with the result in warp 0's buffer 0.
+__device__ __forceinline__ void gs_cta_merge(unsigned char* smem, int W, int kcap, int K) {
+  const int warp = threadIdx.x >> 5;
+  for (int st = 1; st < W; st <<= 1) {
+    __syncthreads();
+    if ((warp % (2 * st)) == 0 && warp + st < W) {
+      GsWarpView a = gs_view(smem, warp, kcap), b = gs_view(smem, warp + st, kcap);
+      gs_merge2(a.list[0], b.list[0], a.list[1], K);
+      const int lane = threadIdx.x & 31;
+      for (int i = lane; i < K; i += 32) a.list[0][i] = a.list[1][i];
+      __syncwarp();
+    }
+  }
+  __syncthreads();
+}
+
 // The warp's insertion state: threshold (own K-th best, lowered by the row threshold), queue fill,
 // per-thread queue (ablation variant).
 struct GsIns {
@@ -289,16 +330,8 @@ __global__ void __launch_bounds__(kGsMaxWarps * 32) gridselect_kernel(const GsPa
     __syncwarp();
     cur = 0;
   }
-  __syncthreads();
+  gs_cta_merge(gs_smem, W, p.kcap, K);
   if (warp == 0) {
-    // threshold = warp 0's own K-th best: a key of another list can equal the adopted row threshold
-    // (it is that list's K-th best) and must not be rejected
-    s.thr = w.list[cur][K - 1];
-    for (int ow = 1; ow < W; ++ow) {
-      const GsWarpView o = gs_view(gs_smem, ow, p.kcap);
-      for (int b = 0; b < K; b += 32) gs_insert<0>(w, cur, K, (b + lane < K) ? o.list[0][b + lane] : kGsInf, s, nullptr);
-    }
-    gs_drain<0>(w, cur, K, s);
     unsigned long long* cand = p.cand + ((size_t)row * p.G + cta) * K;
     for (int i = lane; i < K; i += 32) cand[i] = w.list[cur][i];
   }
@@ -325,14 +358,8 @@ __global__ void __launch_bounds__(kGsMaxWarps * 32) gridselect_kernel(const GsPa
     __syncwarp();
     cur = 0;
   }
-  __syncthreads();
+  gs_cta_merge(gs_smem, W, p.kcap, K);
   if (warp == 0) {
-    s.thr = w.list[cur][K - 1];
-    for (int ow = 1; ow < W; ++ow) {
-      const GsWarpView o = gs_view(gs_smem, ow, p.kcap);
-      for (int b = 0; b < K; b += 32) gs_insert<0>(w, cur, K, (b + lane < K) ? o.list[0][b + lane] : kGsInf, s, nullptr);
-    }
-    gs_drain<0>(w, cur, K, s);
     U* ov = (U*)p.out_vals + row * p.k;
     int64_t* oi = p.out_idx + row * p.k;
     for (int i = lane; i < K; i += 32) {
