@@ -251,6 +251,9 @@ def main():
                     help="key type (f32: the paper's; others: the config's f32 keys converted)")
     ap.add_argument("--window", type=int, default=0, help="sample-guided window: 0 auto, 1 on, -1 off (ablation)")
     ap.add_argument("--tma", type=int, default=0, help="bulk-copy streaming: 0 auto, 1 on, -1 off (ablation)")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p"],
+                    help="split-row candidate exchange: one NCCL all-gather, or peer stores over CUDA IPC "
+                         "(PeerExchange, SURVEY §8(f) NEXT #2)")
     ap.add_argument("--dist-backend", default="nccl", help="nccl (default); gloo only to self-test the "
                     "multi-rank flow with several ranks on one GPU")
     args = ap.parse_args()
@@ -332,7 +335,13 @@ def main():
                                                                                   mbits)), dtype=torch.uint8, device=dev)
         mout = (torch.empty(k, dtype=kdt, device=dev), torch.empty(k, dtype=torch.int64, device=dev))
 
+    if split and args.exchange == "p2p":
+        pex = atdist.PeerExchange(k, kdt, dev)
+
     def step(events=None):
+        if split and args.exchange == "p2p":
+            return atdist.select_split_row_p2p(xd.reshape(-1), k, total_len, rank * n, pex, workspace=ws_shard,
+                                               merge_workspace=ws_merge, out=mout)
         if split:
             return atdist.select_split_row(
                 xd.reshape(-1), k, total_len=total_len, shard_offset=rank * n, buffers=gbuf,
@@ -423,6 +432,7 @@ def main():
             "dtype": args.dtype, "data": "synthetic",
             "config": {"workload": cfg, "batch": c["batch"], "n": n, "k": k, "dist": c["dist"], "select": "min",
                        "per_gpu_rows": batch, "split_row": split,
+                       "exchange": (args.exchange if split else None),
                        "l2": "input (%.2f GB) larger than L2 (126 MB): no flush needed" % (in_bytes / 1e9)
                        if in_bytes > (256 << 20) else "input smaller than L2: consecutive steps may hit L2",
                        "parallelism": f"{'split-row' if split else ('rows' if cfg == 'c2' else 'replica')}x{world}"},

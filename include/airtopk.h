@@ -204,6 +204,31 @@ airtopk_status airtopk_select_shard(const void* keys, airtopk_dtype dtype, int64
 /* Index width of the merge select: bits of total_len + world * k - 1 (0 on invalid arguments). */
 int airtopk_merge_idx_bits(int64_t total_len, int world, int64_t k);
 
+/* Collective-fused split-row exchange over peer memory:
+ * the NCCL all-gather replaced by direct stores into every rank's gather buffers (CUDA IPC; P2P over
+ * NVLink / NVSwitch). Set-up (once per buffer set): each rank exports its gather buffers and flag
+ * array with airtopk_ipc_handle (a 64-byte handle + the offset of the pointer inside its allocation),
+ * the handles are exchanged out of band (e.g. torch.distributed all_gather_object), and every rank
+ * opens its peers' with airtopk_ipc_open (and later airtopk_ipc_close). Per call, with a fresh
+ * nonzero epoch (the same on every rank, e.g. a call counter):
+ *   airtopk_shard_push   one launch: this rank's k values + global indices (from
+ *                        airtopk_select_shard) are stored into slot `rank` of EVERY rank's gather
+ *                        buffers (peer_vals[r] / peer_idx[r], r < world, this rank's own included),
+ *                        then this rank's flag (peer_flags[r][rank]) is set to epoch in every rank
+ *                        after all its stores are visible (system-scope fence + release store);
+ *                        `ticket` is one zeroed device word owned by this rank (reset by the kernel);
+ *   airtopk_wait_flags   one-CTA launch that returns once flags[0..world) all equal epoch (acquire);
+ *                        the merge select enqueued after it sees every rank's entries.
+ * Values are raw key bits of `dtype`, indices int64, buffers [world * k] on each rank's device. */
+airtopk_status airtopk_ipc_handle(const void* dev_ptr, void* handle_out, uint64_t* offset_out);
+airtopk_status airtopk_ipc_open(const void* handle, uint64_t offset, void** dev_ptr_out);
+airtopk_status airtopk_ipc_close(void* dev_ptr);
+airtopk_status airtopk_shard_push(const void* vals, const int64_t* idx, int64_t k, airtopk_dtype dtype, int world,
+                                  int rank, void* const* peer_vals, int64_t* const* peer_idx,
+                                  uint32_t* const* peer_flags, uint32_t epoch, uint32_t* ticket,
+                                  airtopk_stream_t stream);
+airtopk_status airtopk_wait_flags(const uint32_t* flags, int world, uint32_t epoch, airtopk_stream_t stream);
+
 /* End-to-end convenience with HOST buffers: copies keys host->device, selects, copies the results
  * device->host and SYNCHRONISES `stream` before returning. Pinned (page-locked) host memory gives
  * asynchronous DMA; pageable memory works but is staged by the driver. Device staging (keys,

@@ -25,7 +25,8 @@ EXPORTS = (
     "airtopk_select_u32", "airtopk_workspace_bytes_with_idx", "airtopk_select_with_idx",
     "airtopk_select_host", "airtopk_status_str", "airtopk_last_cuda_error", "airtopk_version",
     "airtopk_describe", "airtopk_select_with_idx_ex", "airtopk_workspace_bytes_shard", "airtopk_select_shard",
-    "airtopk_merge_idx_bits",
+    "airtopk_merge_idx_bits", "airtopk_ipc_handle", "airtopk_ipc_open", "airtopk_ipc_close", "airtopk_shard_push",
+    "airtopk_wait_flags",
 )
 
 
@@ -97,6 +98,16 @@ def load(path: str = LIB_PATH):
     lib.airtopk_select_shard.restype = ci
     lib.airtopk_merge_idx_bits.argtypes = [i64, ci, i64]
     lib.airtopk_merge_idx_bits.restype = ci
+    lib.airtopk_ipc_handle.argtypes = [vp, vp, ctypes.POINTER(ctypes.c_uint64)]
+    lib.airtopk_ipc_handle.restype = ci
+    lib.airtopk_ipc_open.argtypes = [vp, ctypes.c_uint64, ctypes.POINTER(vp)]
+    lib.airtopk_ipc_open.restype = ci
+    lib.airtopk_ipc_close.argtypes = [vp]
+    lib.airtopk_ipc_close.restype = ci
+    lib.airtopk_shard_push.argtypes = [vp, vp, i64, ci, ci, ci, vp, vp, vp, ctypes.c_uint32, vp, vp]
+    lib.airtopk_shard_push.restype = ci
+    lib.airtopk_wait_flags.argtypes = [vp, ci, ctypes.c_uint32, vp]
+    lib.airtopk_wait_flags.restype = ci
     lib.airtopk_select_host.argtypes = [vp, ci, i64, i64, i64, ci, vp, vp, vp]
     lib.airtopk_select_host.restype = ci
     lib.airtopk_status_str.argtypes = [ci]

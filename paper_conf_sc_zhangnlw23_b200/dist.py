@@ -90,3 +90,88 @@ def select_split_row(x_shard, k: int, total_len: int, shard_offset: int, largest
     idx_bits = merge_idx_bits(total_len, world, k)
     mfn = merge_fn or (lambda a, b, kq, ib, lg: select_with_idx(a, b, kq, ib, largest=lg))
     return mfn(gv, gi, k, idx_bits, largest)
+
+
+class PeerExchange:
+    """Collective-fused split-row exchange: gather buffers [world * k] and a
+    flag array on every rank, opened by every peer through CUDA IPC (handles exchanged once with
+    all_gather_object over `group`). exchange() = ONE push kernel (this rank's k entries stored into
+    slot `rank` of every rank's buffers, then its flag raised in every rank) + ONE wait kernel (all
+    flags carry this call's epoch) — no NCCL collective. Every rank must call exchange() in the same
+    order (the epoch is a call counter)."""
+
+    def __init__(self, k: int, dtype, device, group=None):
+        import ctypes
+        from . import dtype_code, lib
+        self.lib = lib()
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self.k = k
+        self.dt = dtype_code(dtype)
+        self.vals = torch.empty(self.world * k, dtype=dtype, device=device)
+        self.idx = torch.empty(self.world * k, dtype=torch.int64, device=device)
+        self.flags = torch.zeros(self.world, dtype=torch.int32, device=device)
+        self.ticket = torch.zeros(1, dtype=torch.int32, device=device)
+        torch.cuda.synchronize(device)
+        mine = []
+        for t in (self.vals, self.idx, self.flags):
+            h = (ctypes.c_char * 64)()
+            off = ctypes.c_uint64(0)
+            st = self.lib.airtopk_ipc_handle(t.data_ptr(), h, ctypes.byref(off))
+            if st != 0:
+                raise RuntimeError(f"airtopk_ipc_handle failed ({st})")
+            mine.append((bytes(h), int(off.value)))
+        allh = [None] * self.world
+        dist.all_gather_object(allh, mine, group=group)
+        self.opened = []
+        ptrs = [[], [], []]
+        for r in range(self.world):
+            for b, t in enumerate((self.vals, self.idx, self.flags)):
+                if r == self.rank:
+                    ptrs[b].append(t.data_ptr())
+                    continue
+                hb, off = allh[r][b]
+                p = ctypes.c_void_p()
+                st = self.lib.airtopk_ipc_open((ctypes.c_char * 64).from_buffer_copy(hb), off, ctypes.byref(p))
+                if st != 0:
+                    raise RuntimeError(f"airtopk_ipc_open failed ({st})")
+                self.opened.append(p.value)
+                ptrs[b].append(p.value)
+        arr = lambda xs: (ctypes.c_void_p * self.world)(*xs)
+        self.peer_vals, self.peer_idx, self.peer_flags = arr(ptrs[0]), arr(ptrs[1]), arr(ptrs[2])
+        self.epoch = 0
+        dist.barrier(group=group)
+
+    def slot(self):
+        """(values, indices) views of this rank's slot: the shard select writes here."""
+        s = slice(self.rank * self.k, (self.rank + 1) * self.k)
+        return self.vals[s], self.idx[s]
+
+    def exchange(self, stream=None):
+        self.epoch = (self.epoch + 1) & 0xFFFFFFFF or 1
+        s = (stream if stream is not None else torch.cuda.current_stream(self.vals.device)).cuda_stream
+        v, i = self.slot()
+        st = self.lib.airtopk_shard_push(v.data_ptr(), i.data_ptr(), self.k, self.dt, self.world, self.rank,
+                                         self.peer_vals, self.peer_idx, self.peer_flags, self.epoch,
+                                         self.ticket.data_ptr(), s)
+        if st != 0:
+            raise RuntimeError(f"airtopk_shard_push failed ({st})")
+        st = self.lib.airtopk_wait_flags(self.flags.data_ptr(), self.world, self.epoch, s)
+        if st != 0:
+            raise RuntimeError(f"airtopk_wait_flags failed ({st})")
+
+    def close(self):
+        for p in self.opened:
+            self.lib.airtopk_ipc_close(p)
+        self.opened = []
+
+
+def select_split_row_p2p(x_shard, k: int, total_len: int, shard_offset: int, ex: PeerExchange, largest: bool = False,
+                         workspace=None, merge_workspace=None, out=None):
+    """select_split_row with the exchange over peer memory (PeerExchange) instead of NCCL."""
+    x_shard = x_shard.reshape(-1)
+    pad_base = total_len + ex.rank * k
+    select_shard(x_shard, k, shard_offset, pad_base, largest=largest, out=ex.slot(), workspace=workspace)
+    ex.exchange()
+    return select_with_idx(ex.vals, ex.idx, k, merge_idx_bits(total_len, ex.world, k), largest=largest,
+                           workspace=merge_workspace, out=out)
