@@ -133,6 +133,10 @@ typedef struct {
   uint32_t* status;     /* optional DEVICE word: after the select the library ORs every row's
                            AIRTOPK_ERR_* flags into it (one extra tiny launch; the caller zeroes it and
                            reads it after synchronising). NULL = not collected. Radix engines only. */
+  int32_t sorted;       /* 1: every row's K results come out sorted in the selection order (ascending
+                           keys for select-min, descending for select-max; equal keys by ascending
+                           index) — one extra launch, K <= 4096 (else AIRTOPK_EINVAL). 0 = unordered
+                           (GridSelect rows are always sorted). */
 } airtopk_options;
 
 #define AIRTOPK_TRACE_MAX_PASSES 16
@@ -228,6 +232,19 @@ airtopk_status airtopk_shard_push(const void* vals, const int64_t* idx, int64_t 
                                   uint32_t* const* peer_flags, uint32_t epoch, uint32_t* ticket,
                                   airtopk_stream_t stream);
 airtopk_status airtopk_wait_flags(const uint32_t* flags, int world, uint32_t epoch, airtopk_stream_t stream);
+
+/* The paper's kernel-organisation ablations (§3.1), a plain radix
+ * select with a runtime digit width: design 0 = naive (Fig. 2: histogram, prefix sum, target digit,
+ * filter as four kernels per iteration), 1 = iteration-fused (Fig. 3: filter + histogram in one
+ * kernel, scan in its last block, then a last-filter kernel), 2 = 1 with the last filter fused into the
+ * last iteration. digit_bits 8 or 11. Same results as airtopk_select (lowest-index
+ * ties). Keys of <= 32 bits, len < 2^32, 1 <= k < len, batch <= 65535; workspace from
+ * airtopk_ablation_workspace. *kernels_out (optional) receives the launches enqueued. */
+size_t airtopk_ablation_workspace(airtopk_dtype dtype, int64_t batch, int64_t len, int64_t alpha);
+airtopk_status airtopk_select_ablation(const void* keys, airtopk_dtype dtype, int64_t batch, int64_t len, int64_t k,
+                                       int select_min, void* out_vals, int64_t* out_idx, int design, int digit_bits,
+                                       int64_t alpha, void* workspace, size_t workspace_bytes,
+                                       airtopk_stream_t stream, int* kernels_out);
 
 /* End-to-end convenience with HOST buffers: copies keys host->device, selects, copies the results
  * device->host and SYNCHRONISES `stream` before returning. Pinned (page-locked) host memory gives

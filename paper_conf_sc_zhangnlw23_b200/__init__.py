@@ -60,8 +60,9 @@ def _check(status: int):
 
 
 def _opts(alpha=0, engine=ENGINE_AUTO, ctas_per_row=0, cluster_size=0, trace=None, events=None, window=0, tma=0,
-          early_stop=0, status=None):
+          early_stop=0, status=None, sorted_out=False):
     o = Options()
+    o.sorted = 1 if sorted_out else 0
     o.early_stop = int(early_stop)
     o.window = int(window)
     o.tma = int(tma)
@@ -145,7 +146,7 @@ def _raise_status(st):
 def select(x, k: int, largest: bool = False, *, alpha: int = 0, engine: int = ENGINE_AUTO,
            ctas_per_row: int = 0, cluster_size: int = 0, trace=None, events=None, window: int = 0,
            tma: int = 0, early_stop: int = 0, workspace=None, out=None, stream=None, status=None,
-           check: bool = False):
+           check: bool = False, sorted: bool = False):
     """Top-K of each row of `x` ([batch, len] or [len], contiguous CUDA tensor).
 
     Returns (values, indices): [batch, k] of x.dtype (raw bit copies) and int64 row-local indices,
@@ -153,6 +154,7 @@ def select(x, k: int, largest: bool = False, *, alpha: int = 0, engine: int = EN
     `stream` (default: torch's current stream of x's device); nothing is synchronised unless
     check=True (then the device status word is read back and DeviceError raised if set).
     `status`: optional 1-element int32 CUDA tensor the AIRTOPK_ERR_* bits are OR-ed into.
+    sorted=True: each row comes out in selection order (one extra launch, K <= 4096).
     """
     torch = _torch()
     if not x.is_cuda:
@@ -173,7 +175,7 @@ def select(x, k: int, largest: bool = False, *, alpha: int = 0, engine: int = EN
             _check_out(vals, (batch, k), x2.dtype, dev, "out[0] (values)")
             _check_out(idx, (batch, k), torch.int64, dev, "out[1] (indices)")
         st = _status_word(check, status, dev)
-        o = _opts(alpha, engine, ctas_per_row, cluster_size, trace, events, window, tma, early_stop, st)
+        o = _opts(alpha, engine, ctas_per_row, cluster_size, trace, events, window, tma, early_stop, st, sorted)
         need = int(lib().airtopk_workspace_bytes_ex(dt, batch, length, k, ctypes.byref(o)))
         workspace = _workspace(workspace, need, dev)
         ws_ptr = workspace.data_ptr() if workspace is not None else None
@@ -260,6 +262,29 @@ def select_shard(x_shard, k: int, shard_offset: int, pad_base: int, largest: boo
                                           workspace.data_ptr() if workspace is not None else None,
                                           workspace.numel() if workspace is not None else 0, _stream(stream, dev)))
     return vals, idx
+
+
+def select_ablation(x, k: int, design: int, digit_bits: int = 11, largest: bool = False, alpha: int = 0):
+    """The paper's kernel-organisation ablations (airtopk_select_ablation): design 0 naive (Fig. 2),
+    1 iteration-fused (Fig. 3), 2 fused last filter; digit_bits 8 or 11. Returns
+    (values, indices, kernel launches)."""
+    torch = _torch()
+    x2 = x.reshape(1, -1) if x.dim() == 1 else x
+    if not x2.is_cuda or not x2.is_contiguous():
+        raise ValueError("select_ablation needs a contiguous CUDA tensor")
+    batch, length = x2.shape
+    dt = dtype_code(x2.dtype)
+    dev = x2.device
+    with torch.cuda.device(dev):
+        vals = torch.empty((batch, k), dtype=x2.dtype, device=dev)
+        idx = torch.empty((batch, k), dtype=torch.int64, device=dev)
+        need = int(lib().airtopk_ablation_workspace(dt, batch, length, alpha))
+        ws = torch.empty(max(need, 1), dtype=torch.uint8, device=dev)
+        nk = ctypes.c_int(0)
+        _check(lib().airtopk_select_ablation(x2.data_ptr(), dt, batch, length, k, 0 if largest else 1, vals.data_ptr(),
+                                             idx.data_ptr(), int(design), int(digit_bits), int(alpha), ws.data_ptr(),
+                                             ws.numel(), _stream(None, dev), ctypes.byref(nk)))
+    return vals, idx, int(nk.value)
 
 
 def select_host(x_host, k: int, largest: bool = False, out=None, stream=None):

@@ -26,7 +26,7 @@ EXPORTS = (
     "airtopk_select_host", "airtopk_status_str", "airtopk_last_cuda_error", "airtopk_version",
     "airtopk_describe", "airtopk_select_with_idx_ex", "airtopk_workspace_bytes_shard", "airtopk_select_shard",
     "airtopk_merge_idx_bits", "airtopk_ipc_handle", "airtopk_ipc_open", "airtopk_ipc_close", "airtopk_shard_push",
-    "airtopk_wait_flags",
+    "airtopk_wait_flags", "airtopk_ablation_workspace", "airtopk_select_ablation",
 )
 
 
@@ -43,6 +43,7 @@ class Options(ctypes.Structure):
         ("tma", ctypes.c_int32),
         ("early_stop", ctypes.c_int32),
         ("status", ctypes.c_void_p),
+        ("sorted", ctypes.c_int32),
     ]
 
 
@@ -108,6 +109,11 @@ def load(path: str = LIB_PATH):
     lib.airtopk_shard_push.restype = ci
     lib.airtopk_wait_flags.argtypes = [vp, ci, ctypes.c_uint32, vp]
     lib.airtopk_wait_flags.restype = ci
+    lib.airtopk_ablation_workspace.argtypes = [ci, i64, i64, i64]
+    lib.airtopk_ablation_workspace.restype = sz
+    lib.airtopk_select_ablation.argtypes = [vp, ci, i64, i64, i64, ci, vp, vp, ci, ci, i64, vp, sz, vp,
+                                            ctypes.POINTER(ci)]
+    lib.airtopk_select_ablation.restype = ci
     lib.airtopk_select_host.argtypes = [vp, ci, i64, i64, i64, ci, vp, vp, vp]
     lib.airtopk_select_host.restype = ci
     lib.airtopk_status_str.argtypes = [ci]

@@ -313,6 +313,7 @@ static airtopk_status validate(const SelectArgs& a) {
   if (a.window < -1 || a.window > 1) return AIRTOPK_EINVAL;
   if (a.early_stop < -1 || a.early_stop > 0) return AIRTOPK_EINVAL;
   if (a.in_idx && (a.batch != 1 || a.idx_bits < 1 || a.idx_bits > 63)) return AIRTOPK_EINVAL;
+  if (a.sorted < 0 || a.sorted > 1 || (a.sorted && a.k > kSortMaxK)) return AIRTOPK_EINVAL;
   return AIRTOPK_OK;
 }
 
@@ -335,6 +336,7 @@ static airtopk_status run(const SelectArgs& a, void* ws, size_t ws_bytes, cudaSt
   Plan p = make_plan(a);
   if (p.engine == 3) {
     cudaError_t e = run_trivial(a, s);
+    if (e == cudaSuccess && a.sorted) e = run_sort_rows(a, s);
     return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
   }
   if (!ws || ws_bytes < p.bytes) return AIRTOPK_ENOSPACE;
@@ -350,6 +352,7 @@ static airtopk_status run(const SelectArgs& a, void* ws, size_t ws_bytes, cudaSt
                   : (p.engine == 5) ? run_batch(a, p, ws, s)
                   : (p.engine == 6) ? run_resident(a, p, ws, s)
                                     : run_grid(a, p, ws, s);
+  if (e == cudaSuccess && a.sorted) e = run_sort_rows(a, s);
   if (e == cudaSuccess && a.status) e = collect_status(a, p, ws, s);
   return e == cudaSuccess ? AIRTOPK_OK : fail_cuda(e);
 }
@@ -377,6 +380,7 @@ static SelectArgs make_args(const void* keys, int dt, int64_t batch, int64_t len
     a.tma = opt->tma;
     a.early_stop = opt->early_stop;
     a.status = opt->status;
+    a.sorted = opt->sorted;
   }
   if (a.alpha == 0) a.alpha = 128;
   return a;

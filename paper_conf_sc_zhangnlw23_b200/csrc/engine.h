@@ -25,6 +25,7 @@ struct SelectArgs {
   int early_stop = 0;               // 0 on, -1 off (ablation)
   int64_t idx_off = 0;              // added to every output index (airtopk_select_shard)
   unsigned* status = nullptr;       // optional device word: row error flags OR-ed in after the select
+  int sorted = 0;                   // 1: rows sorted in selection order after the select (K <= 4096)
   int64_t* trace = nullptr;
   void* const* events = nullptr;    // optional cudaEvent_t[n_events] recorded around launches
   int n_events = 0;
@@ -92,6 +93,9 @@ cudaError_t run_trivial(const SelectArgs& a, cudaStream_t s);
 // K entries that sort last in the selection order (multi-GPU shard shorter than K): value bits of the
 // maximum code, indices pad_base + j
 cudaError_t run_pad(int kind, int sel_min, void* vals, int64_t* idx, int64_t n, int64_t pad_base, cudaStream_t s);
+// sort every row's K results in selection order (one CTA per row, bitonic in shared memory, K <= 4096)
+cudaError_t run_sort_rows(const SelectArgs& a, cudaStream_t s);
+constexpr int64_t kSortMaxK = 4096;
 // OR the error flags of every row state of a grid / cluster engine workspace into *a.status
 cudaError_t collect_status(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 int grid_blocks_per_sm(const SelectArgs& a, int idx64);

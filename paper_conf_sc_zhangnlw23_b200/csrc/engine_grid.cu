@@ -149,6 +149,75 @@ cudaError_t run_pad(int kind, int sel_min, void* vals, int64_t* idx, int64_t n, 
   return cudaGetLastError();
 }
 
+// Sorted output option: one CTA per row sorts its K (code, index) pairs ascending — bitonic network
+// over the next power of two in shared memory (padding sorts last), values re-derived from the codes.
+template <int KIND>
+__global__ void __launch_bounds__(1024) sort_rows_kernel(typename KT<KIND>::U* ov, int64_t* oi, int64_t k,
+                                                         int sel_min) {
+  using U = typename KT<KIND>::U;
+  extern __shared__ __align__(16) unsigned long long srt[];
+  unsigned long long* sc = srt;               // codes (as 64-bit)
+  unsigned long long* si = srt + kSortMaxK;   // indices
+  const int64_t row = blockIdx.x;
+  int n = 1;
+  while (n < k) n <<= 1;
+  for (int i = threadIdx.x; i < n; i += blockDim.x) {
+    const bool in = i < k;
+    sc[i] = in ? (unsigned long long)to_code<KIND>(ov[row * k + i], sel_min != 0) : ~0ull;
+    si[i] = in ? (unsigned long long)oi[row * k + i] : ~0ull;
+  }
+  __syncthreads();
+  for (int size = 2; size <= n; size <<= 1) {
+    for (int stride = size >> 1; stride > 0; stride >>= 1) {
+      for (int i = threadIdx.x; i < n / 2; i += blockDim.x) {
+        const int a = 2 * i - (i & (stride - 1)), b = a + stride;  // pair (a, b), a's bit `stride` clear
+        const bool up = (a & size) == 0;
+        const unsigned long long ca = sc[a], cb = sc[b], ia = si[a], ib = si[b];
+        const bool gt = ca > cb || (ca == cb && ia > ib);
+        if (gt == up) {
+          sc[a] = cb; sc[b] = ca;
+          si[a] = ib; si[b] = ia;
+        }
+      }
+      __syncthreads();
+    }
+  }
+  for (int i = threadIdx.x; i < k; i += blockDim.x) {
+    ov[row * k + i] = from_code<KIND>((U)sc[i], sel_min != 0);
+    oi[row * k + i] = (int64_t)si[i];
+  }
+}
+
+cudaError_t run_sort_rows(const SelectArgs& a, cudaStream_t s) {
+  const size_t smem = (size_t)2 * kSortMaxK * 8;
+  const unsigned g = (unsigned)a.batch;
+  cudaError_t e = cudaSuccess;
+  switch (a.kind) {
+    case K_F32:
+      if ((e = func_attr(sort_rows_kernel<K_F32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) == cudaSuccess)
+        sort_rows_kernel<K_F32><<<g, 1024, smem, s>>>((uint32_t*)a.out_vals, a.out_idx, a.k, a.sel_min);
+      break;
+    case K_F16:
+      if ((e = func_attr(sort_rows_kernel<K_F16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) == cudaSuccess)
+        sort_rows_kernel<K_F16><<<g, 1024, smem, s>>>((uint16_t*)a.out_vals, a.out_idx, a.k, a.sel_min);
+      break;
+    case K_BF16:
+      if ((e = func_attr(sort_rows_kernel<K_BF16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) == cudaSuccess)
+        sort_rows_kernel<K_BF16><<<g, 1024, smem, s>>>((uint16_t*)a.out_vals, a.out_idx, a.k, a.sel_min);
+      break;
+    case K_F64:
+      if ((e = func_attr(sort_rows_kernel<K_F64>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) == cudaSuccess)
+        sort_rows_kernel<K_F64><<<g, 1024, smem, s>>>((uint64_t*)a.out_vals, a.out_idx, a.k, a.sel_min);
+      break;
+    case K_U32:
+      if ((e = func_attr(sort_rows_kernel<K_U32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) == cudaSuccess)
+        sort_rows_kernel<K_U32><<<g, 1024, smem, s>>>((uint32_t*)a.out_vals, a.out_idx, a.k, a.sel_min);
+      break;
+  }
+  if (e != cudaSuccess) return e;
+  return cudaGetLastError();
+}
+
 __global__ void status_kernel(const RowState* st, int64_t batch, unsigned* status) {
   unsigned e = 0;
   for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < batch; r += (int64_t)gridDim.x * blockDim.x)

@@ -134,3 +134,27 @@ def test_select_on_non_current_device():
     torch.cuda.synchronize(1)
     assert_parity(raw.view(np.uint32), "f32", 1000, True, v.view(torch.int32).cpu().numpy().view(np.uint32),
                   i.cpu().numpy())
+
+
+@pytest.mark.parametrize("engine", [0, 1, 2, 5, 6])
+def test_sorted_output_option(engine):
+    """sorted=True: each row in selection order (keys ascending for select-min / descending for
+    select-max, equal keys by ascending index), identical set to the oracle."""
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    batch, n, k = 40, 1 << 17, 3000
+    raw = gen.adversarial_f32(81, batch * n, m_bits=22).reshape(batch, n)
+    x = torch.from_numpy(raw).cuda()
+    for largest in (False, True):
+        try:
+            v, i = at.select(x, k, largest=largest, engine=engine, sorted=True)
+        except at.AirTopKError:
+            assert engine in (5, 6)  # shape not eligible for that engine
+            continue
+        torch.cuda.synchronize()
+        vb, ii = v.cpu().numpy(), i.cpu().numpy()
+        assert_parity(raw.view(np.uint32), "f32", k, not largest, vb.view(np.uint32), ii)
+        rv, ri = oracle.topk_sort(raw, k, select_min=not largest)   # canonical (code, index) order
+        assert np.array_equal(ii, ri) and np.array_equal(vb.view(np.uint32), rv.view(np.uint32))
+    with pytest.raises(at.AirTopKError):
+        at.select(x, 4097, sorted=True)
