@@ -67,13 +67,13 @@ def main():
             n = int(rng.integers(300, 1 << 17))
         else:
             n = int(rng.integers(1 << 17, 1 << 21))
-        batch = int(rng.choice([1, 1, 1, 2, 3, 7, 33])) if n < (1 << 20) else 1
+        batch = int(rng.choice([1, 1, 1, 2, 3, 7, 33, 150])) if n < (1 << 18) else int(rng.choice([1, 1, 4, 20]))
         k = int(rng.choice([1, 2, max(1, n // 1000), max(1, n // 10), n // 2 + 1, n, int(rng.integers(1, n + 1))]))
         k = max(1, min(k, n))
         sm = bool(rng.integers(0, 2))
         kw = {}
-        engine = int(rng.choice([0, 0, 1, 2, 4]))
-        if engine == 4 and (dtn == "f64" or k > 256):
+        engine = int(rng.choice([0, 0, 1, 2, 4, 5, 6, 7]))
+        if engine in (4, 7) and (dtn == "f64" or k > 2048):
             engine = 0
         if engine:
             kw["engine"] = engine
@@ -83,12 +83,31 @@ def main():
             kw["alpha"] = int(rng.choice([1, 4, 128, 1 << 40]))
         if rng.random() < 0.2:
             kw["early_stop"] = -1
-        if engine == 2 and rng.random() < 0.5:
+        if engine in (2, 6) and rng.random() < 0.5:
             kw["cluster_size"] = int(rng.choice([1, 2, 4, 8, 16]))
+        if rng.random() < 0.1 and k <= 4096:
+            kw["sorted"] = True
+        abl = rng.random() < 0.05 and dtn != "f64" and k < n
         raw, pat = make_keys(rng, dtn, batch, n)
         cases += 1
         try:
-            v, i = gpu_select(raw, dtn, k, sm, **kw)
+            if abl:  # the paper's kernel organisations (ablation harness)
+                import torch
+                import paper_conf_sc_zhangnlw23_b200 as at
+                from helpers import to_bits, to_device
+                design, b = int(rng.integers(0, 3)), int(rng.choice([8, 11]))
+                kw = {"ablation": (design, b)}
+                vv, ii, _ = at.select_ablation(to_device(raw, dtn), k, design, b, largest=not sm)
+                torch.cuda.synchronize()
+                v, i = to_bits(vv, dtn), ii.cpu().numpy()
+            else:
+                try:
+                    v, i = gpu_select(raw, dtn, k, sm, **kw)
+                except Exception as e:  # an engine the shape is not eligible for: AIRTOPK_EINVAL
+                    if kw.get("engine") in (5, 6) and "EINVAL" in str(e):
+                        cases -= 1
+                        continue
+                    raise
             assert_parity(raw, dtn, k, sm, v, i)
         except Exception as e:  # noqa: BLE001
             fails += 1

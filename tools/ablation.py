@@ -81,3 +81,42 @@ for w, name in ((-1, "paper's passes (window off)"), (0, "default (window)")):
     t = per_launch(x, 2048, window=w)
     s = sum(t)
     print(f"{name}: total {s:.1f} us |", " ".join(f"{v:.1f} ({100 * v / s:.2f}%)" for v in t))
+
+print()
+print("# Kernel organisation (P:146-156, airtopk_select_ablation: plain kernels, scalar loads): us per select")
+print("# design 0 naive (Fig. 2: 4 kernels per iteration), 1 iteration-fused (Fig. 3), 2 fused last filter (P:156)")
+
+
+def timed_abl(x, k, design, b, reps=10):
+    for _ in range(2):
+        at.select_ablation(x, k, design, b)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(reps):
+        _, _, nk = at.select_ablation(x, k, design, b)
+    e1.record()
+    e1.synchronize()
+    return e0.elapsed_time(e1) / reps * 1e3, nk
+
+
+print(f"{'data':>12} {'N':>6} {'K':>6} " + " ".join(f"{nm:>22}" for nm in
+      ("naive b=8", "naive b=11", "fused b=8", "fused b=11", "fused+lastfilter b=11")))
+for dist, m in (("uniform", 20), ("adversarial", 20)):
+    for lg in (20, 26, 28):
+        n = 1 << lg
+        x = torch.from_numpy(gen.keys(dist, 905, n, m_bits=m).reshape(1, n)).cuda()
+        k = 2048
+        cells = []
+        for design, b in ((0, 8), (0, 11), (1, 8), (1, 11), (2, 11)):
+            t, nk = timed_abl(x, k, design, b)
+            cells.append(f"{t:>12.1f} ({nk:2d} kern)")
+        print(f"{dist:>12} 2^{lg:<4} {k:>6} " + " ".join(f"{c:>22}" for c in cells), flush=True)
+        del x
+        torch.cuda.empty_cache()
+
+print()
+print("# Sorted output option (one extra launch): us per select, batch 100 x 2^20 normal")
+x = torch.from_numpy(gen.normal_f32(906, 100 << 20).reshape(100, 1 << 20)).cuda()
+for k in (32, 256, 4096):
+    print(f"K {k:5d}: unordered {timed(x, k):8.1f}  sorted {timed(x, k, sorted=True):8.1f}", flush=True)
