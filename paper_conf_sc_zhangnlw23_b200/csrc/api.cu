@@ -273,7 +273,8 @@ static void choose_launch(const SelectArgs& a, Plan& p) {
   }
   // batch 1 (no trace, no tail): every pass after the window pass in one cooperative launch
   // (window = -1 keeps the paper's one-kernel-per-pass structure: the P:146-156 ablations)
-  p.fused = (p.engine == 1 && a.batch == 1 && !a.in_idx && a.trace == nullptr && !p.tail && a.window >= 0 &&
+  p.fused = (p.engine == 1 && a.batch == 1 && !a.in_idx && (a.trace == nullptr || getenv("AIRTOPK_TAIL_STAMPS")) &&
+             !p.tail && a.window >= 0 &&
              getenv("AIRTOPK_NO_FUSED") == nullptr) ? 1 : 0;
   // bulk-copy streaming for a few long rows (every SM busy with 1 CTA); register loads otherwise
   p.tma = 0;

@@ -78,6 +78,8 @@ cudaError_t run_grid(const SelectArgs& a, const Plan& pl, void* ws, cudaStream_t
   gp.early_stop = a.early_stop;
   gp.idx_off = a.idx_off;
   gp.thist = base + pl.off_thist;
+  gp.tstamp = nullptr;
+  if (a.trace && getenv("AIRTOPK_TAIL_STAMPS")) gp.tstamp = a.trace;  // debug (tools/tail_stamps.py)
   gp.tcnt = (unsigned long long*)(base + pl.off_tcnt);
   {
     static const char* env2 = getenv("AIRTOPK_SMALL_FINISH");  // A/B knob (0 = off)

@@ -72,6 +72,7 @@ struct GridParams {
   int small_finish;  // a buffer-source pass over <= this many entries finishes the row in one CTA
   int early_stop;   // 0 on, -1 off (ablation)
   int64_t idx_off;  // added to every output index (airtopk_select_shard)
+  int64_t* tstamp;  // fused tail debug: per pass [run_pass done, barrier passed, scan done] (CTA 0)
   void* thist;      // fused tail (batch 1): 3 rotating global histograms
   unsigned long long* tcnt;  // fused tail: candidates stored by pass q (zeroed with the state)
 };
@@ -897,7 +898,16 @@ __device__ __forceinline__ bool tail_pass(const GridParams& p, int q, TailState&
     for (int i = tid; i < kHistSlots * HC; i += kBlock) sh_hist[i] = 0;
     __syncthreads();
   }
+  auto tst = [&](int f) {
+    if (p.tstamp && blockIdx.x == 0 && tid == 0 && q < 16) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      p.tstamp[q * 4 + f] = (int64_t)t;
+    }
+  };
+  tst(0);
   run_pass<KIND, IdxT, DF, DH, false, kBlock, 0, false, kGridBU>(c);
+  tst(1);
   if (!(c.do_hist || DF == 0)) return true;  // emit-all pass: the row is complete
   __syncthreads();
   CountT* gh = (CountT*)p.thist + (size_t)(q % 3) * kMaxBins;
@@ -909,8 +919,10 @@ __device__ __forceinline__ bool tail_pass(const GridParams& p, int q, TailState&
     if (v) atomicAdd(&gh[i], (CountT)v);
   }
   cg::this_grid().sync();  // every CTA's histogram, results and candidates of pass q are published
+  tst(2);
   const ScanResult r = scan_choose<kBlock>([&](int b) { return (unsigned long long)__ldcg(&gh[b]); }, nb, S.K, sh_tmp,
                                            sh_res);
+  tst(3);
   if (blockIdx.x == 0) {
     CountT* gz = (CountT*)p.thist + (size_t)((q + 2) % 3) * kMaxBins;
     for (int i = tid; i < kMaxBins; i += kBlock) gz[i] = 0;

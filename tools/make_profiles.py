@@ -19,7 +19,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, os.path.join(ROOT, "tools"))
 import ncu_summary  # noqa: E402
 
-OUT = os.path.join(ROOT, "gpurun_out")
+OUT = os.path.join(ROOT, "gpurun_out")  # (a sub-directory may be given as the 2nd argument)
 PROF = os.path.join(ROOT, "profiles")
 
 KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum", "dram__sectors_read.sum",
@@ -30,10 +30,12 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "smsp__average_warp_latency_issue_stalled_long_scoreboard.pct", "sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active"]
 
 
-def main(rnd):
+def main(rnd, out=OUT):
+    global OUT
+    OUT = out
     os.makedirs(PROF, exist_ok=True)
-    tpath = os.path.join(PROF, "traffic_launches.json")
-    traffic = json.load(open(tpath)) if os.path.exists(tpath) else {}  # merged: configs not re-measured stay
+    tpath = os.path.join(PROF, "traffic.json")
+    traffic = json.load(open(tpath)) if os.path.exists(tpath) else {}  # merged: plans not re-measured stay
     for f in sorted(glob.glob(os.path.join(OUT, "launches_*.csv"))):
         cfg = os.path.basename(f)[len("launches_"):-4]
         try:
@@ -52,7 +54,11 @@ def main(rnd):
             lines.append(f"{i:3d} {ncu_summary.short(d['name'])[:50]:50s} {t:9.1f} {rd / 1e6:12.1f} {wr / 1e6:13.1f}")
             per.setdefault(i, rd + wr)
         open(os.path.join(PROF, f"{rnd}_launches_{cfg}.txt"), "w").write("\n".join(lines) + "\n")
-        traffic[cfg] = {str(k): v for k, v in per.items()}
+        side = os.path.join(OUT, f"plan_{cfg}.json")  # written by prof_select.py --plan-out
+        if os.path.exists(side):
+            pk = json.load(open(side))
+            traffic[pk["plan_key"]] = {"launches_per_select": pk["launches_per_select"],
+                                       "bytes": [per[i] for i in sorted(per)], "source": f"{rnd}_launches_{cfg}.txt"}
     for f in sorted(glob.glob(os.path.join(OUT, "*.ncu-rep"))):
         name = os.path.basename(f)[:-8]
         raw = subprocess.run(["ncu", "-i", f, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
@@ -73,9 +79,9 @@ def main(rnd):
         txt = open(f).read().strip()
         if txt:
             open(os.path.join(PROF, f"{rnd}_{os.path.basename(f)}"), "w").write(txt.splitlines()[-1] + "\n")
-    json.dump(traffic, open(os.path.join(PROF, "traffic_launches.json"), "w"), indent=1)
+    json.dump(traffic, open(tpath, "w"), indent=1)
     print("wrote", sorted(os.listdir(PROF)))
 
 
 if __name__ == "__main__":
-    main(sys.argv[1] if len(sys.argv) > 1 else "r01")
+    main(sys.argv[1] if len(sys.argv) > 1 else "r02", sys.argv[2] if len(sys.argv) > 2 else OUT)
