@@ -191,7 +191,7 @@ def select(x, k: int, largest: bool = False, *, alpha: int = 0, engine: int = EN
 
 
 def select_with_idx(x, in_idx, k: int, idx_bits: int, largest: bool = False, workspace=None, stream=None,
-                    out=None, status=None, check: bool = False):
+                    out=None, status=None, check: bool = False, engine: int = ENGINE_AUTO):
     """Merge select over one row whose elements carry index VALUES in_idx (int64, distinct, <
     2^idx_bits); ties rank by in_idx value; returned indices are in_idx values."""
     torch = _torch()
@@ -215,7 +215,7 @@ def select_with_idx(x, in_idx, k: int, idx_bits: int, largest: bool = False, wor
         need = int(lib().airtopk_workspace_bytes_with_idx(dt, n, k, idx_bits))
         workspace = _workspace(workspace, need, dev)
         st = _status_word(check, status, dev)
-        o = _opts(status=st)
+        o = _opts(engine=engine, status=st)
         _check(lib().airtopk_select_with_idx_ex(x.data_ptr(), in_idx.data_ptr(), idx_bits, dt, n, k,
                                                 0 if largest else 1, vals.data_ptr(), idx.data_ptr(),
                                                 workspace.data_ptr() if workspace is not None else None,

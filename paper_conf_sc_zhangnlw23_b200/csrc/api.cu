@@ -185,6 +185,9 @@ Plan make_plan(const SelectArgs& a) {
 // and small rows, the grid engine (one launch per pass, whole GPU per row) for long rows.
 static int auto_engine(const SelectArgs& a) {
   if (a.window > 0 && !a.in_idx) return 1;  // window requested: grid window pass (+ cluster tail)
+  // split-row merges of >= 2^18 gathered candidates: the grid passes (tools/merge_ab.py: 8 x 2^16
+  // candidates 46 us vs 61 us in one cluster)
+  if (a.in_idx && a.len >= (int64_t(1) << 18)) return 1;
   if (a.len <= (int64_t(1) << 19)) return 2;  // one launch: measured fastest from 2^17 to 2^19 keys per row
   return 1;
 }

@@ -28,6 +28,8 @@
 #include "device.cuh"
 #include "engine.h"
 #include "finish.cuh"
+#include "passes.cuh"
+#include "tma.cuh"
 
 namespace airtopk {
 
@@ -69,7 +71,7 @@ __device__ __forceinline__ void rstamp(const ResidentParams& p, int f) {
 
 template <typename W>
 struct ResShared {
-  unsigned hist[2][kMaxBins];  // this CTA's histogram of the current pass (read remotely)
+  unsigned hist[2][kMaxBins + 32];  // this CTA's histogram of the current pass (read remotely) + dummy bin
   SelScratch<W, kRWarps> sel;
   unsigned long long tmp[kRWarps];
   ScanResult res;
@@ -165,6 +167,7 @@ __global__ void __launch_bounds__(kRBlock, 1) resident_kernel(const ResidentPara
       const unsigned hm = (1u << dh.width) - 1u, fm = (1u << df.width) - 1u;
       unsigned* hist = sh.hist[q & 1];
       for (int i = tid; i < (1 << dh.width); i += kRBlock) hist[i] = 0;
+      if (tid == 0) hist[kMaxBins] = 0;
       __syncthreads();
       const W tc = (W)(tcode >> df.shift), bc = tc & ~(W)fm;
       const unsigned ti = (unsigned)(tidx >> df.shift), bi = ti & ~fm;
@@ -188,7 +191,11 @@ __global__ void __launch_bounds__(kRBlock, 1) resident_kernel(const ResidentPara
           }
         }
         if (__any_sync(kFull, win)) emit(win, code, idx);
-        if (cand) atomicAdd(&hist[dh.is_idx ? (idx >> dh.shift) & hm : (unsigned)((W)code >> dh.shift) & hm], 1u);
+        // red.shared.add (equal addresses in a warp are aggregated by the hardware); non-candidates
+        // hit the dummy bin instead of branching (passes.cuh)
+        const unsigned d = cand ? (dh.is_idx ? (idx >> dh.shift) & hm : (unsigned)((W)code >> dh.shift) & hm)
+                                : (unsigned)kMaxBins;
+        shared_inc(smem_addr(hist) + 4u * d);
       }
       rstamp(p, 2 + 3 * min(q, 2));
       cl.sync();  // every CTA's histogram of digit q is complete

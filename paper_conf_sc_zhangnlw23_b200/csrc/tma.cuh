@@ -99,8 +99,16 @@ __device__ __forceinline__ bool mbar_try_wait_hint(unsigned bar, unsigned parity
   return ok != 0;
 }
 
+#ifndef AIRTOPK_MBAR_HINT
+#define AIRTOPK_MBAR_HINT 1
+#endif
 __device__ __forceinline__ void mbar_wait_sleep(unsigned bar, unsigned parity) {
-  while (!mbar_try_wait_hint(bar, parity)) {
+  if (AIRTOPK_MBAR_HINT) {
+    while (!mbar_try_wait_hint(bar, parity)) {
+    }
+  } else {
+    while (!mbar_try_wait(bar, parity)) {
+    }
   }
 }
 
