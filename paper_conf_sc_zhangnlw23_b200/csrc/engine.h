@@ -83,8 +83,14 @@ cudaError_t run_batch(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t
 cudaError_t run_resident(const SelectArgs& a, const Plan& p, void* ws, cudaStream_t s);
 // batched engine constants shared with the host plan (engine_batch.cuh)
 constexpr int kBatchBlock = 1024, kBatchWarps = 32;
-constexpr int kBatchSlotWarps = 16;  // warps per consumer group = (chunk, warp) slots per chunk
-constexpr int kBatchStage = 32768;   // bytes per chunk (one bulk-copy ring stage)
+#ifndef AIRTOPK_BATCH_GROUPS
+#define AIRTOPK_BATCH_GROUPS 4        // phase-B consumer warp groups (take ring stages in turn)
+#endif
+#ifndef AIRTOPK_BATCH_STAGE_BYTES
+#define AIRTOPK_BATCH_STAGE_BYTES 24576
+#endif
+constexpr int kBatchSlotWarps = 32 / AIRTOPK_BATCH_GROUPS;  // warps per consumer group = slots per chunk
+constexpr int kBatchStage = AIRTOPK_BATCH_STAGE_BYTES;      // bytes per chunk (one bulk-copy ring stage)
 constexpr int kBatchFcap = 16384;    // entries (results + window members) one row may stage in the finish
 // resident-cluster engine (engine_resident.cuh)
 constexpr int kResidentCap = 32768;  // keys per CTA held in shared memory (<= 4-byte keys; half for 8-byte)

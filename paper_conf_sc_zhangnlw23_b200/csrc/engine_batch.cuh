@@ -50,15 +50,20 @@ constexpr int kBBlock = kBatchBlock;          // threads per CTA (1 CTA per SM)
 constexpr int kBWarps = kBBlock / 32;
 static_assert(kBWarps == kBatchWarps, "host/device slot geometry");
 constexpr unsigned kBStage = kBatchStage;     // bytes per bulk-copy ring stage = one chunk of a row
-constexpr int kBStages = 6;                   // ring depth: 192 KiB in flight per SM
+#ifndef AIRTOPK_BATCH_STAGES
+#define AIRTOPK_BATCH_STAGES 8
+#endif
+constexpr int kBStages = AIRTOPK_BATCH_STAGES;  // ring depth: 8 x 24 KiB = 192 KiB in flight per SM
 constexpr int kBPre = 4;                      // stages issued before the sampling phase
 #ifndef AIRTOPK_BATCH_L2PRE
 #define AIRTOPK_BATCH_L2PRE 0  // measured: L2 prefetches during phase A slow the sampling, stream unchanged
 #endif
 constexpr int kBL2Pre = AIRTOPK_BATCH_L2PRE;  // further chunks per CTA prefetched into L2 during phase A
-// Phase B consumers: two groups of 16 warps take alternate stages, 4 vectors per thread each (a
-// warp's per-stage overhead — barrier wait, count store, loop — is amortised over 2 KiB).
-constexpr int kBGroups = 2;
+// Phase B consumers: four groups of 8 warps take the stages in turn, 6 vectors per thread each (a
+// warp's per-stage overhead — barrier wait, count store, loop — is amortised over 3 KiB; measured on
+// c2: 4 x 8 warps on 8 x 24 KiB stages stream at 6.6 TB/s, 2 x 16 on 6 x 32 KiB at 6.1, 1 x 32 on
+// 6 x 32 KiB at 5.3).
+constexpr int kBGroups = AIRTOPK_BATCH_GROUPS;
 constexpr int kBGWarps = kBWarps / kBGroups;
 constexpr int kBGThreads = kBGWarps * 32;
 constexpr int kBVT = (int)(kBStage / 16 / kBGThreads);  // 16-byte vectors per thread per stage
