@@ -96,7 +96,7 @@ typedef enum {
                                    keys of <= 32 bits, len < 2^32 and K <= 2048, else
                                    AIRTOPK_EINVAL. Rows come out sorted. Never chosen by AUTO. */
   AIRTOPK_ENGINE_BATCH = 5,     /* batched rows in ONE cooperative launch: per-row sample window,
-                                   single read of every row into fixed per-(chunk, warp) slots,
+                                   single read of every row into fixed per-chunk slots,
                                    per-row shared-memory finish; rows whose window fails are redone
                                    by a cluster-engine launch. Needs 16-byte aligned rows and a
                                    window that fits 16K entries per row, else AIRTOPK_EINVAL. */

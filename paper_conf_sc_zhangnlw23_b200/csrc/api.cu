@@ -163,13 +163,16 @@ Plan make_plan(const SelectArgs& a) {
     const double per_row = rhi / (double)ns * (double)a.len;  // expected entries <= hi
     if (ns >= 1024 && rhi < (double)(ns - 1) && per_row <= 0.5 * kBatchFcap) {
       const int64_t chunk = kBatchStage / es;
-      const double e_slot = (double)(kBatchStage / 16) * vec / kBatchSlotWarps * rhi / (double)ns;
+      const double e_slot = (double)(kBatchStage / 16) * vec * rhi / (double)ns;  // expected entries per chunk
       p.batch_ok = 1;
       p.bnsamp = (int)ns;
       p.cpc = (int)((a.len + chunk - 1) / chunk);
-      p.nwc = p.cpc * kBatchSlotWarps;
-      // multiple of 16 entries: slots start on 32-byte sectors (the writers pad to whole sectors)
-      p.scap = (int)align_up((size_t)std::ceil(e_slot + 6.0 * std::sqrt(e_slot) + 8.0), 16);
+      p.nwc = p.cpc;  // one slot per chunk (shared by the consumer group's warps)
+      // the true count below hi can be ~2x the estimate (hi is a sample order statistic of rank
+      // ~rhi: relative spread ~1/sqrt(rhi)), plus a 6-sigma Poisson margin per chunk; a multiple of
+      // 16 entries: slots start on 32-byte sectors (the group leader pads to whole sectors)
+      const double e2 = 2.0 * e_slot;
+      p.scap = (int)align_up((size_t)std::ceil(e2 + 6.0 * std::sqrt(e2) + 8.0), 16);
       const size_t nslot = (size_t)a.batch * p.nwc;
       p.off_bcnt = p.bytes;
       p.off_bslot = p.off_bcnt + align_up(nslot * 2, 256);

@@ -53,7 +53,7 @@ struct Plan {
   int batch_ok;      // the shape qualifies (alignment is checked at run time)
   int bnsamp;        // samples per row
   int cpc;           // 32 KiB chunks per row
-  int nwc;           // (chunk, warp) slots per row
+  int nwc;           // slots per row (one per chunk)
   int scap;          // entries per slot
   int rslice;        // resident-cluster engine: keys per CTA
   size_t off_state, off_hist, off_thist, off_tcnt, off_bcode, off_bidx, off_samp, off_bcnt, off_bslot, off_bsidx,
@@ -89,7 +89,6 @@ constexpr int kBatchBlock = 1024, kBatchWarps = 32;
 #ifndef AIRTOPK_BATCH_STAGE_BYTES
 #define AIRTOPK_BATCH_STAGE_BYTES 24576
 #endif
-constexpr int kBatchSlotWarps = 32 / AIRTOPK_BATCH_GROUPS;  // warps per consumer group = slots per chunk
 constexpr int kBatchStage = AIRTOPK_BATCH_STAGE_BYTES;      // bytes per chunk (one bulk-copy ring stage)
 constexpr int kBatchFcap = 16384;    // entries (results + window members) one row may stage in the finish
 // resident-cluster engine (engine_resident.cuh)

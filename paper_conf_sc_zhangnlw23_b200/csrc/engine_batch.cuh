@@ -17,8 +17,9 @@
 //      stages (cp.async.bulk, TMA engine, mbarrier full/empty handshake: 192 KiB in flight per SM,
 //      the first 4 issued before phase A). Per element ONE compare of the raw key bits against the
 //      transformed threshold hi (exact); the rare flagged keys (code <= hi) are written by their
-//      warp to a FIXED slot of its (chunk, warp) — no atomics, no queues, no block barriers in the
-//      streaming loop — and the warp stores the slot's count.
+//      warp to the FIXED slot of the chunk at an offset from ONE shared atomic per flagged warp —
+//      no global atomics, no queues, no block barriers in the streaming loop — and the group
+//      leader stores the slot's count once the group released the stage.
 //   C  finish: CTA r gathers its row's slots (prefix sum over the slot counts) into shared memory
 //      and registers, checks that the window holds the K-th key (R < K <= R + W, R = #codes < lo,
 //      W = #members), emits the R results, then selects the K - R smallest members by radix passes
@@ -69,7 +70,6 @@ constexpr int kBGThreads = kBGWarps * 32;
 constexpr int kBVT = (int)(kBStage / 16 / kBGThreads);  // 16-byte vectors per thread per stage
 static_assert(kBVT * 16 * kBGThreads == (int)kBStage, "stage = group threads x kBVT vectors");
 static_assert(kBStages % kBGroups == 0, "a stage always belongs to the same group");
-static_assert(kBGWarps == kBatchSlotWarps, "host/device slot geometry");
 constexpr int kBFcap = kBatchFcap;            // entries (results + members) one row may stage in the finish
 constexpr size_t kBRingBytes = (size_t)kBStages * kBStage;
 static_assert((size_t)kMaxSamples * 4 <= (size_t)(kBStages - kBPre) * kBStage, "samples fit the unused stages");
@@ -83,10 +83,10 @@ struct BatchParams {
   int64_t* out_idx;
   int64_t idx_off;
   RowState* st;
-  unsigned short* cnt;    // [batch][nwc] entries written per (chunk, group warp) slot (cap + 1 = overflow)
+  unsigned short* cnt;    // [batch][nwc] entries written per chunk slot (cap + 1 = overflow)
   void* scode;            // [batch][nwc][scap] codes
   unsigned* sidx;         // [batch][nwc][scap] row indices
-  int nwc;                // slots per row = chunks per row * kBGWarps
+  int nwc;                // slots per row = chunks per row
   int scap;               // entries per slot
   int cpc;                // chunks per row
   int nsamp;              // samples per row
@@ -255,7 +255,7 @@ __device__ __forceinline__ void batch_prefetch_l2(const BatchParams& p, int64_t 
                : "memory");
 }
 
-// The input is read exactly once: its L2 lines are marked evict-first so the (chunk, warp) slots
+// The input is read exactly once: its L2 lines are marked evict-first so the chunk slots
 // written meanwhile stay in L2 for the finish.
 template <typename U>
 __device__ __forceinline__ void batch_issue(const BatchParams& p, int64_t ch, unsigned ring, int stage) {
@@ -279,7 +279,7 @@ __device__ __forceinline__ void batch_issue(const BatchParams& p, int64_t ch, un
 // one min of the raw bits; the flags are only built when the minimum hits (a few lanes per stage).
 template <int KIND, bool FULL>
 __device__ __forceinline__ void batch_classify(const BatchParams& p, int64_t row, int ci, unsigned long long hi,
-                                               unsigned sbase, int nv, int gt, int gw) {
+                                               unsigned sbase, int nv, int gt, unsigned* scnt) {
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
   constexpr int VEC = 16 / sizeof(U);
@@ -301,8 +301,7 @@ __device__ __forceinline__ void batch_classify(const BatchParams& p, int64_t row
       m = (valid && t < m) ? t : m;
     }
   }
-  const size_t slot = (size_t)row * p.nwc + (size_t)ci * kBGWarps + gw;
-  int total = 0;
+  const size_t slot = (size_t)row * p.nwc + (size_t)ci;  // the chunk's slot (shared by the group's warps)
   if (__any_sync(kFull, m <= whi)) {
     FlagT fl = 0;
 #pragma unroll
@@ -319,20 +318,16 @@ __device__ __forceinline__ void batch_classify(const BatchParams& p, int64_t row
       const int y = __shfl_up_sync(kFull, incl, o);
       if (lane >= o) incl += y;
     }
-    total = __shfl_sync(kFull, incl, 31);
-    int pos = incl - n;
+    const int total = __shfl_sync(kFull, incl, 31);
+    // the warp's range of the chunk slot: ONE shared atomic on the stage's counter (the group
+    // leader stores the slot count once every warp of the group has released the stage)
+    unsigned wb = 0;
+    if (lane == 31) wb = atomicAdd(scnt, (unsigned)total);
+    int pos = (int)__shfl_sync(kFull, wb, 31) + incl - n;
     U* sc = (U*)p.scode + slot * p.scap;
     unsigned* si = p.sidx + slot * p.scap;
     const U xmask = sel_min ? (U)0 : (U)~(U)0;
-    // pad the written entries to whole 32-byte sectors: a partially written L2 sector would have to
-    // be filled from DRAM when the finish reads it (measured: ~7 us of the finish)
-    constexpr int kSec = 32 / (sizeof(U) < 4 ? sizeof(U) : 4);
-    const int padded = min(p.scap, (total + kSec - 1) / kSec * kSec);
     const unsigned long long keep = l2_policy_evict_last();
-    for (int q = total + lane; q < padded; q += 32) {
-      st_keep(sc + q, (U)0, keep);
-      st_keep(si + q, 0u, keep);
-    }
 #pragma unroll 1
     while (fl) {
       const int b = ((sizeof(FlagT) == 8) ? __ffsll((long long)fl) : __ffs((int)fl)) - 1;
@@ -350,7 +345,27 @@ __device__ __forceinline__ void batch_classify(const BatchParams& p, int64_t row
       ++pos;
     }
   }
-  if (lane == 0) st_keep(p.cnt + slot, (unsigned short)(total > p.scap ? p.scap + 1 : total), l2_policy_evict_last());
+}
+
+// Group leader, after every warp of its group released the stage: store the chunk slot's count
+// (cap + 1 = overflow) and pad the written entries to whole 32-byte sectors (a partially written
+// L2 sector would have to be filled from DRAM when the finish reads it; measured ~7 us), then
+// reset the stage's counter for its next chunk.
+template <typename U>
+__device__ __forceinline__ void batch_slot_done(const BatchParams& p, int64_t row, int ci, unsigned* scnt) {
+  const unsigned c = *(volatile unsigned*)scnt;
+  *scnt = 0;
+  const size_t slot = (size_t)row * p.nwc + (size_t)ci;
+  const unsigned long long keep = l2_policy_evict_last();
+  constexpr int kSec = 32 / (sizeof(U) < 4 ? sizeof(U) : 4);
+  const int padded = min(p.scap, ((int)c + kSec - 1) / kSec * kSec);
+  U* sc = (U*)p.scode + slot * p.scap;
+  unsigned* si = p.sidx + slot * p.scap;
+  for (int q = (int)c; q < padded; ++q) {
+    st_keep(sc + q, (U)0, keep);
+    st_keep(si + q, 0u, keep);
+  }
+  st_keep(p.cnt + slot, (unsigned short)((int)c > p.scap ? p.scap + 1 : (int)c), keep);
 }
 
 // ---------------------------------------------------------------------------------- phase C
@@ -358,7 +373,7 @@ __device__ __forceinline__ void batch_classify(const BatchParams& p, int64_t row
 template <int KIND>
 __device__ void batch_finish_row(const BatchParams& p, int64_t row, void* stage,
                                  BatchShared<std::conditional_t<sizeof(typename KT<KIND>::U) == 8, unsigned long long,
-                                                                unsigned>>& sh) {
+                                                                unsigned>>& sh, bool dry = false) {
   using U = typename KT<KIND>::U;
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
   constexpr int WB = 8 * (int)sizeof(W);
@@ -381,10 +396,13 @@ __device__ void batch_finish_row(const BatchParams& p, int64_t row, void* stage,
   bstamp(p, 20);
   U* stc = (U*)stage;
   unsigned* sti = (unsigned*)((char*)stage + (size_t)kBFcap * sizeof(U));
-  // --- gather: warp w takes slots w*32 + lane + r*kBBlock (coalesced counts, loaded for kGR
-  // rounds at once), a warp scan places its slots' entries, ONE shared atomic per warp and round
-  // reserves staging room (the order of entries is irrelevant to the selection), and every entry
-  // load of a round is in flight together ---
+  // --- gather: warp w takes the contiguous slot range [w*spw, (w+1)*spw) (one chunk slot per
+  // lane, coalesced counts), a warp scan places its slots' entries, ONE shared atomic per warp
+  // reserves staging room (the order of entries is irrelevant to the selection), then the warp's
+  // entries are loaded lane-parallel (entry e -> slot lane by a shuffle binary search over the
+  // inclusive slot prefix): consecutive lanes read consecutive entries of a slot, and every load
+  // of a batch is in flight before its stores (the staging pointer is generic: interleaved
+  // stores would serialise the loads) ---
   const int nwc = p.nwc;
   const unsigned short* cnt = p.cnt + (size_t)row * nwc;
   if (tid == 0) {
@@ -393,62 +411,50 @@ __device__ void batch_finish_row(const BatchParams& p, int64_t row, void* stage,
   }
   __syncthreads();
   bstamp(p, 21);
-  // per warp iteration: kGR slots per lane; offsets first (scans + one shared atomic per round),
-  // then every entry load of the iteration, then the stores — the staging pointer is generic, so
-  // interleaved stores would serialise the loads (measured: ~5 us)
-  constexpr int kGR = 2, kGJ = 4;
+  constexpr int kGJ = 4;  // entries per lane per batch
+  const int spw = (nwc + kBWarps - 1) / kBWarps;
+  const int s_end = min(nwc, (warp + 1) * spw);
 #pragma unroll 1
-  for (int base = warp * 32 + lane; base - lane < nwc; base += kGR * kBBlock) {
-    int cc[kGR];
-    unsigned o[kGR];
+  for (int s0 = warp * spw; s0 < s_end; s0 += 32) {
+    const int sl = s0 + lane;
+    int cc = sl < s_end ? (int)__ldcg(cnt + sl) : 0;
+    if (cc > p.scap) sh.bad = 1;
+    cc = min(cc, p.scap);
+    int incl = cc;
 #pragma unroll
-    for (int r = 0; r < kGR; ++r) {
-      const int sl = base + r * kBBlock;
-      cc[r] = sl < nwc ? (int)__ldcg(cnt + sl) : 0;
+    for (int q = 1; q < 32; q <<= 1) {
+      const int y = __shfl_up_sync(kFull, incl, q);
+      if (lane >= q) incl += y;
     }
+    const int all = __shfl_sync(kFull, incl, 31);
+    unsigned b = 0;
+    if (lane == 0 && all) b = atomicAdd(&sh.cnt, (unsigned)all);
+    b = __shfl_sync(kFull, b, 0);
+    bstamp(p, 22);
+#pragma unroll 1
+    for (int e0 = 0; e0 < all; e0 += 32 * kGJ) {
+      U vc[kGJ];
+      unsigned vi[kGJ];
 #pragma unroll
-    for (int r = 0; r < kGR; ++r) {
-      if (cc[r] > p.scap) sh.bad = 1;
-      cc[r] = min(cc[r], p.scap);
-      int incl = cc[r];
+      for (int t = 0; t < kGJ; ++t) {
+        const int e = e0 + t * 32 + lane;
+        int L = 0;  // number of slot lanes whose inclusive prefix is <= e: e's slot
 #pragma unroll
-      for (int q = 1; q < 32; q <<= 1) {
-        const int y = __shfl_up_sync(kFull, incl, q);
-        if (lane >= q) incl += y;
-      }
-      const int tot = __shfl_sync(kFull, incl, 31);
-      unsigned b = 0;
-      if (lane == 0 && tot) b = atomicAdd(&sh.cnt, (unsigned)tot);
-      o[r] = __shfl_sync(kFull, b, 0) + (unsigned)(incl - cc[r]);
-    }
-    U vc[kGR][kGJ];
-    unsigned vi[kGR][kGJ];
-#pragma unroll
-    for (int r = 0; r < kGR; ++r) {
-      const size_t src = ((size_t)row * nwc + base + r * kBBlock) * p.scap;
-#pragma unroll
-      for (int j = 0; j < kGJ; ++j) {
-        if (j < cc[r]) {
-          vc[r][j] = __ldcg((const U*)p.scode + src + j);
-          vi[r][j] = __ldcg(p.sidx + src + j);
+        for (int h = 16; h > 0; h >>= 1)
+          if (__shfl_sync(kFull, incl, L + h - 1) <= e) L += h;
+        const int ex = __shfl_sync(kFull, incl - cc, L);
+        if (e < all) {
+          const size_t src = ((size_t)row * nwc + s0 + L) * p.scap + (e - ex);
+          vc[t] = __ldcg((const U*)p.scode + src);
+          vi[t] = __ldcg(p.sidx + src);
         }
       }
-    }
 #pragma unroll
-    for (int r = 0; r < kGR; ++r) {
-#pragma unroll
-      for (int j = 0; j < kGJ; ++j) {
-        if (j < cc[r] && o[r] + j < (unsigned)kBFcap) {
-          stc[o[r] + j] = vc[r][j];
-          sti[o[r] + j] = vi[r][j];
-        }
-      }
-      const size_t src = ((size_t)row * nwc + base + r * kBBlock) * p.scap;
-#pragma unroll 1
-      for (int j = kGJ; j < cc[r]; ++j) {
-        if (o[r] + j < (unsigned)kBFcap) {
-          stc[o[r] + j] = __ldcg((const U*)p.scode + src + j);
-          sti[o[r] + j] = __ldcg(p.sidx + src + j);
+      for (int t = 0; t < kGJ; ++t) {
+        const unsigned d = b + (unsigned)(e0 + t * 32 + lane);
+        if (e0 + t * 32 + lane < all && d < (unsigned)kBFcap) {
+          stc[d] = vc[t];
+          sti[d] = vi[t];
         }
       }
     }
@@ -456,6 +462,7 @@ __device__ void batch_finish_row(const BatchParams& p, int64_t row, void* stage,
   }
   __syncthreads();
   bstamp(p, 7);
+  if (dry) return;  // (debug: gather only)
   const int n = (int)sh.cnt;
   if (sh.bad || n > kBFcap || n < (int)p.k) {
     fail();  // slot overflow / too many entries / fewer than K keys up to hi
@@ -528,6 +535,7 @@ __global__ void __launch_bounds__(kBBlock, 1) batch_kernel(const BatchParams p) 
   using W = std::conditional_t<sizeof(U) == 8, unsigned long long, unsigned>;
   extern __shared__ __align__(128) unsigned char batch_smem[];
   __shared__ BatchShared<W> sh;
+  __shared__ unsigned sh_scnt[kBStages];  // entries of the chunk in each ring stage (its chunk slot)
   cg::grid_group grid = cg::this_grid();
   const int G = (int)gridDim.x, cta = (int)blockIdx.x, tid = threadIdx.x;
   const unsigned ring = smem_addr(batch_smem);
@@ -536,6 +544,7 @@ __global__ void __launch_bounds__(kBBlock, 1) batch_kernel(const BatchParams p) 
   const int64_t mine = cta < nch ? (nch - 1 - cta) / G + 1 : 0;  // chunks cta, cta + G, ...
   bstamp(p, 0);
   // the first kBPre chunks this CTA streams start landing in the ring while the rows are sampled
+  if (tid < kBStages) sh_scnt[tid] = 0;
   if (tid == 0) {
     if (cta == 0) *p.fail = 0;  // (appends happen after the first grid barrier)
     for (int i = 0; i < kBStages; ++i) {
@@ -566,7 +575,7 @@ __global__ void __launch_bounds__(kBBlock, 1) batch_kernel(const BatchParams p) 
     for (int i = kBPre; i < kBStages && i < mine; ++i) batch_issue<U>(p, cta + (int64_t)i * G, ring, i);
   }
   {
-    const int grp = (tid >> 5) / kBGWarps, gt = tid & (kBGThreads - 1), gw = gt >> 5;
+    const int grp = (tid >> 5) / kBGWarps, gt = tid & (kBGThreads - 1);
     const int64_t rb = p.len * (int64_t)sizeof(U);
     // chunk cta + i*G = (row, ci), advanced incrementally by 2 iterations; the next chunk's window is
     // loaded one iteration ahead (its L2 latency must not sit in front of every chunk)
@@ -601,16 +610,20 @@ __global__ void __launch_bounds__(kBBlock, 1) batch_kernel(const BatchParams p) 
       const int64_t left = rb - ci * (int64_t)kBStage;
       mbar_wait_sleep(fullb + 8u * st, ph);
       if (ws == 1) {
-        if (left >= (int64_t)kBStage) batch_classify<KIND, true>(p, row, ci, hi, ring + st * kBStage, 0, gt, gw);
-        else batch_classify<KIND, false>(p, row, ci, hi, ring + st * kBStage, (int)(left / 16), gt, gw);
+        if (left >= (int64_t)kBStage) batch_classify<KIND, true>(p, row, ci, hi, ring + st * kBStage, 0, gt, &sh_scnt[st]);
+        else batch_classify<KIND, false>(p, row, ci, hi, ring + st * kBStage, (int)(left / 16), gt, &sh_scnt[st]);
       }
       __syncwarp();
       if ((tid & 31) == 0) mbar_arrive(emptyb + 8u * st);
-      // the group leader refills the stage with the chunk kBStages iterations ahead
-      if (gt == 0 && i + kBStages < mine) {
+      // the group leader, once every warp of the group released the stage: the chunk slot's count,
+      // then the refill with the chunk kBStages iterations ahead
+      if (gt == 0) {
         mbar_wait_sleep(emptyb + 8u * st, ph);
-        fence_proxy_async_smem();
-        batch_issue<U>(p, cta + (i + kBStages) * G, ring, st);
+        batch_slot_done<U>(p, row, ci, &sh_scnt[st]);
+        if (i + kBStages < mine) {
+          fence_proxy_async_smem();
+          batch_issue<U>(p, cta + (i + kBStages) * G, ring, st);
+        }
       }
       st += kBGroups;
       if (st >= kBStages) {
@@ -635,6 +648,10 @@ __global__ void __launch_bounds__(kBBlock, 1) batch_kernel(const BatchParams p) 
   grid.sync();
   bstamp(p, 6);
   // ---- C: finish every row (staging in the ring: every bulk copy has been consumed) ----
+#ifdef AIRTOPK_BATCH_FINISH_TWICE  // debug: a first gather-only run (warm instruction cache), stamps overwritten
+  for (int64_t row = cta; row < p.batch; row += G) batch_finish_row<KIND>(p, row, batch_smem, sh, true);
+  __syncthreads();
+#endif
   for (int64_t row = cta; row < p.batch; row += G) batch_finish_row<KIND>(p, row, batch_smem, sh);
   bstamp(p, 15);
 }

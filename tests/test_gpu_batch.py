@@ -1,5 +1,5 @@
 """GPU parity of the batched engine (engine 5, csrc/engine_batch.cuh): one cooperative launch per
-batch — sample, single-read window stream into fixed (chunk, warp) slots, per-row finish — plus the
+batch — sample, single-read window stream into fixed per-chunk slots, per-row finish — plus the
 cluster-engine fallback launch for rows whose window failed. Every output is compared with the CPU
 oracle (identical value bits, identical index set under the lowest-index rule). White-box checks
 read the per-row outcome (RowState.win_state: 4 = finished by the batch kernel, 3 = fallback) from
@@ -83,7 +83,7 @@ def test_batch_ties_and_special_values():
 
 
 def test_batch_slot_overflow_falls_back():
-    """A contiguous run of tiny keys floods a few (chunk, warp) slots: those rows must take the
+    """A contiguous run of tiny keys floods a few chunk slots: those rows must take the
     fallback launch and still be exact; the other rows finish in the batch kernel."""
     batch, n, k = 16, 1 << 20, 256
     raw = gen.uniform_f32(34, batch * n).reshape(batch, n).copy()
