@@ -259,16 +259,16 @@ static void choose_launch(const SelectArgs& a, Plan& p) {
   // read of L they save (tools/engine_ab.py: 1 x 2^22 keys 36 us without vs 51 us with the window,
   // 1 x 2^24 63 vs 73 us, 100 x 2^20 with K = 32768 334 vs 723 us); the paper's passes run instead
   if (a.window == 0 && a.engine == 0 && a.len < (int64_t(1) << 26) && !a.in_idx) p.nsamp = 0;
-  // expected window size per row (entries) -> tail mode for small windows
+  // Cluster tail (one cluster-engine launch runs every pass after the window pass) for small windows:
+  // opt-in only (AIRTOPK_CLUSTER_TAIL=1, A/B). Measured (tools/probe_tail.py, profiles/r02_probe_tail.txt):
+  // on well-behaved rows it equals the fused cooperative tail (batch 1) or the grid passes
+  // (batches), but a window that misses or is rejected restarts the row inside one cluster — a
+  // constant 2^26-key row with K = 10 took 2.68 ms there vs 0.36 ms on the grid.
   p.tail = 0;
-  if (p.nsamp > 0 && a.window >= 0) {
+  if (p.nsamp > 0 && a.window >= 0 && getenv("AIRTOPK_CLUSTER_TAIL") != nullptr) {
     const double f = (double)a.k / (double)a.len, r = f * p.nsamp;
     const double rhi = r + 4.0 * std::sqrt(r * (1.0 - f)) + 9.0;  // sample_kernel's margin
     const double expect = rhi / p.nsamp * (double)a.len;
-    // small windows: one cluster-engine launch runs every pass after the window pass. (Measured: a
-    // tail CTA needs ~25 us per pass at ~20K window entries, where the 444-CTA grid passes are
-    // faster, so the tail is kept for windows of <= 4K entries per CTA of a cluster of <= 16;
-    // tail_q > 0 — grid passes first, then the tail — is supported but off.)
     if (a.engine == 0 && expect <= 16.0 * kTailPerCTA) {
       p.tail = 1;
       p.tail_q = 0;

@@ -312,16 +312,34 @@ def test_window_fallback(case, engine):
 
 @pytest.mark.parametrize("dist,batch,n,k", [("normal", 100, 1 << 20, 256), ("adversarial", 3, 1 << 22, 5000),
                                             ("uniform", 7, 1 << 19, 1), ("uniform", 2, 1 << 21, 20000)])
-def test_window_tail(dist, batch, n, k):
-    """grid engine window pass + one cluster-engine launch finishing every row (tail mode; AUTO
-    sends batches to the batched engine, window=1 asks for the grid engine's window pass)"""
+@pytest.mark.parametrize("cluster_tail", [False, True])
+def test_window_tail(dist, batch, n, k, cluster_tail, monkeypatch):
+    """grid engine window pass (window=1: AUTO sends batches to the batched engine) followed by the
+    grid passes, or — opt-in, AIRTOPK_CLUSTER_TAIL=1 — by one cluster-engine launch finishing
+    every row (tail mode)"""
     import torch
     import paper_conf_sc_zhangnlw23_b200 as at
-    assert at.describe(torch.float32, batch, n, k, window=1)["launches"] == 3
+    if cluster_tail:
+        monkeypatch.setenv("AIRTOPK_CLUSTER_TAIL", "1")
+        assert at.describe(torch.float32, batch, n, k, window=1)["launches"] == 3
     x = _keys(dist, 33, batch, n)
     for sm in (True, False):
         v, i = gpu_select(x, "f32", k, sm, window=1)
         assert_parity(x, "f32", k, sm, v, i)
+
+
+def test_cluster_tail_off_by_default_and_miss_safe():
+    """AUTO never picks the cluster tail (a rejected window restarted the row inside
+    one cluster); a constant row with a tiny K — the window is rejected — runs on the grid and stays
+    exact"""
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    n = 1 << 26
+    d = at.describe(torch.float32, 1, n, 10)
+    assert d["engine"] == 1 and d["cluster_size"] == 0
+    x = np.full((1, n), 0.5, np.float32)
+    v, i = gpu_select(x, "f32", 10, True)
+    assert_parity(x, "f32", 10, True, v, i)
 
 
 def test_window_describe():

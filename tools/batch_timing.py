@@ -38,7 +38,7 @@ mx = lambda f, a=rel: float(np.nanmax(a[:, f]))
 print(f"rows={rows} n={n} k={k} {dist} {'L2 flushed' if do_flush else 'no flush'}")
 print(f"  A sample : loads {med(1):.2f}  select done {med(2):.2f}  end {med(3):.2f} (max {mx(3):.2f}) us")
 print("  A select internals: hist " + " ".join(f"{med(16 + i):.2f}" for i in range(5)))
-print(f"  barrier 1: {mx(4):.2f} | B stream end first/median/last {np.nanmin(rel[:,5]):.2f}/{np.nanmedian(rel[:,5]):.2f}/{mx(5):.2f} | barrier 2 {mx(6):.2f}")
+print(f"  barrier 1: {mx(4):.2f} | B stream end first/median/last {np.nanmin(rel[:,5]):.2f}/{np.nanmedian(rel[:,5]):.2f}/{mx(5):.2f} | C start (max) {mx(6):.2f}")
 print("  C gather internals (start, counts zeroed, offsets, warp 0 entries): "
       + " ".join(f"{med(20 + i):.2f}" for i in range(4)) + f" (max {mx(23):.2f})")
 print(f"  C finish : counts {med(7):.2f}  gather {med(8):.2f}  check {med(9):.2f}  results {med(10):.2f}  "
