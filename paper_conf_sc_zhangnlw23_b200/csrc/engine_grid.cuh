@@ -130,6 +130,14 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
   RowState* st = p.st + row;
+  // Window pass over bulk copies: the ring's first stages (input keys only: nothing the sample kernel
+  // writes) are requested BEFORE the PDL wait, so they stream in while the sample kernel finishes.
+  // (The keys' producer completed before the sample kernel passed its own wait and triggered us.)
+  int pre_issued = 0;
+  if constexpr (DF == 3 && TMA)
+    pre_issued = tma_prologue<typename KT<KIND>::U, HC, kBlock>((const typename KT<KIND>::U*)p.keys + row * p.len,
+                                                                p.len, cta, p.cpr, false,
+                                                                smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>());
   pdl_wait();     // the previous pass's scan (row state, buffers) is complete and visible
   pdl_trigger();  // the next pass may be scheduled as our CTAs retire (hides launch latency)
 
@@ -138,7 +146,13 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   if (FILTER && stop1 != 0 && stop1 - 1 < q - 1) return;  // finished by an earlier early stop
   if (FILTER && q < st->npass) return;                     // digit done by the window pass (digit skip)
   const int win_state = (DF == 3 || (DF == 0 && redo)) ? st->win_state : 0;
-  if (DF == 3 && win_state != 1) return;                   // no window: pass 0 will read L
+  if (DF == 3 && win_state != 1) {                         // no window: pass 0 will read L
+    if constexpr (TMA) {  // the pre-issued copies must land before the CTA's shared memory is released
+      const unsigned fullb = smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>() + tma_stages<HC>() * kTmaChunk;
+      for (int i = 0; i < pre_issued; ++i) mbar_wait(fullb + 8u * i, 0);
+    }
+    return;
+  }
   if (DF == 0 && redo && win_state == 1) return;           // pass 0 was done by the window pass
   const int src1 = FILTER ? st->src1 : 0;    // Alg1 L7-8 (reading 6)
   const int sslot = (src1 == 1) ? 1 : 0;                   // candidate buffer this pass writes
@@ -198,6 +212,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.err = &st->error;
   c.hist = sh_hist;
   c.ring = smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>();
+  c.pre = (DF == 3 && TMA);
   c.wq = &sh_wq[HAS_Q ? warp : 0];
 
   if constexpr (FILTER && DH != 0) {

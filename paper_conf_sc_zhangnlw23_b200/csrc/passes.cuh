@@ -164,6 +164,7 @@ template <typename U, typename IdxT>
 struct PassCtx {
   int q;
   bool emit_all, do_hist, srcL, store, sel_min, reverse;
+  bool pre = false;  // TMA: the ring's first stages were issued before the PDL wait (window pass)
   Digit dh, df;
   Digit dh2;        // DF == 3: the digit after dh (its member histogram at counter offset kHistSlots)
   unsigned long long tcode, tidx;  // fixed prefix bits after scan q-1
@@ -559,7 +560,7 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
       const int64_t cstep = c.reverse ? -(int64_t)c.nslices : (int64_t)c.nslices;
       const uint4* const src0 = vp + c0 * CV;
       const int64_t sstep = cstep * CV;  // in 16-byte vectors
-      tma_prologue<U, HC, BLOCK>(c.rowp, c.len, c.slice, c.nslices, c.reverse, ring);
+      if (!c.pre) tma_prologue<U, HC, BLOCK>(c.rowp, c.len, c.slice, c.nslices, c.reverse, ring);
       __syncthreads();
       int st = 0, pst = NST - 1;    // stage of this / the previous iteration
       unsigned ph = 0, pph = 1;     // their phase parities
