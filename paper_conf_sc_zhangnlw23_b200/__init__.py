@@ -8,6 +8,7 @@ There is no CPU fallback: calling without the built library or on a CPU tensor r
 """
 from __future__ import annotations
 
+import contextlib
 import ctypes
 
 from . import _lib
@@ -45,22 +46,53 @@ def _torch():
     return torch
 
 
+_DTYPES = None
+_NULLCTX = contextlib.nullcontext()
+
+
 def dtype_code(dtype) -> int:
-    torch = _torch()
-    m = {torch.float32: _lib.F32, torch.float16: _lib.F16, torch.bfloat16: _lib.BF16,
-         torch.float64: _lib.F64, torch.uint32: _lib.U32}
-    if dtype not in m:
+    global _DTYPES
+    if _DTYPES is None:
+        torch = _torch()
+        _DTYPES = {torch.float32: _lib.F32, torch.float16: _lib.F16, torch.bfloat16: _lib.BF16,
+                   torch.float64: _lib.F64, torch.uint32: _lib.U32}
+    c = _DTYPES.get(dtype)
+    if c is None:
         raise TypeError(f"unsupported key dtype {dtype} (f32/f16/bf16/f64/u32)")
-    return m[dtype]
+    return c
 
 
 def _check(status: int):
     if status != OK:
+        if status in (_lib.EINVAL, _lib.EDTYPE, _lib.ENOSPACE):
+            raise _lib.AirTopKArgumentError(status, lib())
         raise AirTopKError(status, lib())
+
+
+_OPTS_CACHE = {}
 
 
 def _opts(alpha=0, engine=ENGINE_AUTO, ctas_per_row=0, cluster_size=0, trace=None, events=None, window=0, tma=0,
           early_stop=0, status=None, sorted_out=False):
+    if trace is None and events is None and status is None:
+        # pointer-free options are immutable once built: one ctypes struct per distinct tuple (the
+        # per-call cost of the binding matters for latency-bound rows: c1 is ~12 us on the GPU)
+        key = (alpha, engine, ctas_per_row, cluster_size, window, tma, early_stop, sorted_out)
+        o = _OPTS_CACHE.get(key)
+        if o is None:
+            o = _OPTS_CACHE[key] = _build_opts(*key)
+        return o
+    o = _build_opts(alpha, engine, ctas_per_row, cluster_size, window, tma, early_stop, sorted_out)
+    o.trace = trace.data_ptr() if trace is not None else None
+    o.status = status.data_ptr() if status is not None else None
+    if events is not None:
+        # events: a ctypes array of cudaEvent_t handles (see make_event_array)
+        o.events = ctypes.cast(events, ctypes.c_void_p)
+        o.n_events = len(events)
+    return o
+
+
+def _build_opts(alpha, engine, ctas_per_row, cluster_size, window, tma, early_stop, sorted_out):
     o = Options()
     o.sorted = 1 if sorted_out else 0
     o.early_stop = int(early_stop)
@@ -70,12 +102,6 @@ def _opts(alpha=0, engine=ENGINE_AUTO, ctas_per_row=0, cluster_size=0, trace=Non
     o.engine = int(engine)
     o.ctas_per_row = int(ctas_per_row)
     o.cluster_size = int(cluster_size)
-    o.trace = trace.data_ptr() if trace is not None else None
-    o.status = status.data_ptr() if status is not None else None
-    if events is not None:
-        # events: a ctypes array of cudaEvent_t handles (see make_event_array)
-        o.events = ctypes.cast(events, ctypes.c_void_p)
-        o.n_events = len(events)
     return o
 
 
@@ -103,14 +129,15 @@ def describe(dtype, batch: int, length: int, k: int, alpha: int = 0, engine: int
 
 def _stream(stream, device):
     torch = _torch()
-    s = stream if stream is not None else torch.cuda.current_stream(device)
-    if s.device != device:
-        raise ValueError(f"stream of {s.device} used with tensors on {device}")
-    return s.cuda_stream
+    if stream is None:  # the raw cudaStream_t of torch's current stream (no Stream object built)
+        return torch._C._cuda_getCurrentRawStream(device.index)
+    if stream.device != device:
+        raise ValueError(f"stream of {stream.device} used with tensors on {device}")
+    return stream.cuda_stream
 
 
 def _check_out(t, shape, dtype, device, what):
-    if tuple(t.shape) != tuple(shape) or t.dtype != dtype or t.device != device or not t.is_contiguous():
+    if t.shape != shape or t.dtype != dtype or t.device != device or not t.is_contiguous():
         raise ValueError(f"{what} must be a contiguous {dtype} tensor of shape {tuple(shape)} on {device} "
                          f"(got {t.dtype} {tuple(t.shape)} on {t.device}, contiguous={t.is_contiguous()})")
 
@@ -166,7 +193,9 @@ def select(x, k: int, largest: bool = False, *, alpha: int = 0, engine: int = EN
     batch, length = x2.shape
     dt = dtype_code(x2.dtype)
     dev = x2.device
-    with torch.cuda.device(dev):
+    # the library queries and launches on the current device: make it x's (skipped when it already
+    # is: the context manager costs a few microseconds per call)
+    with (_NULLCTX if dev.index == torch.cuda.current_device() else torch.cuda.device(dev)):
         if out is None:
             vals = torch.empty((batch, k), dtype=x2.dtype, device=dev)
             idx = torch.empty((batch, k), dtype=torch.int64, device=dev)
@@ -176,13 +205,17 @@ def select(x, k: int, largest: bool = False, *, alpha: int = 0, engine: int = EN
             _check_out(idx, (batch, k), torch.int64, dev, "out[1] (indices)")
         st = _status_word(check, status, dev)
         o = _opts(alpha, engine, ctas_per_row, cluster_size, trace, events, window, tma, early_stop, st, sorted)
-        need = int(lib().airtopk_workspace_bytes_ex(dt, batch, length, k, ctypes.byref(o)))
-        workspace = _workspace(workspace, need, dev)
+        L = lib()
+        if workspace is None:
+            workspace = _workspace(None, int(L.airtopk_workspace_bytes_ex(dt, batch, length, k, ctypes.byref(o))), dev)
+        elif workspace.dtype != torch.uint8 or workspace.device != dev or not workspace.is_contiguous():
+            raise ValueError(f"workspace must be a contiguous uint8 tensor on {dev}")
+        # (a caller workspace that is too small is rejected by the library: AIRTOPK_ENOSPACE)
         ws_ptr = workspace.data_ptr() if workspace is not None else None
         ws_bytes = workspace.numel() if workspace is not None else 0
         s = _stream(stream, dev)
-        _check(lib().airtopk_select_ex(x2.data_ptr(), dt, batch, length, k, 0 if largest else 1,
-                                       vals.data_ptr(), idx.data_ptr(), ws_ptr, ws_bytes, s, ctypes.byref(o)))
+        _check(L.airtopk_select_ex(x2.data_ptr(), dt, batch, length, k, 0 if largest else 1,
+                                   vals.data_ptr(), idx.data_ptr(), ws_ptr, ws_bytes, s, ctypes.byref(o)))
         if check:
             _raise_status(st)
     if squeeze:

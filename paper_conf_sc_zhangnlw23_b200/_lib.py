@@ -69,6 +69,11 @@ class AirTopKError(RuntimeError):
         self.status = status
 
 
+class AirTopKArgumentError(AirTopKError, ValueError):
+    """AIRTOPK_EINVAL / EDTYPE / ENOSPACE: the call's arguments (e.g. a caller workspace that is too
+    small) were rejected before anything was enqueued."""
+
+
 def load(path: str = LIB_PATH):
     if not os.path.exists(path):
         raise ImportError(f"{path} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "

@@ -89,7 +89,11 @@ __global__ void __launch_bounds__(kCBlock, 1) cluster_kernel(const ClusterParams
   const unsigned long long kk = (unsigned long long)p.k;
   const unsigned long long cap = (unsigned long long)p.cap_rule;
 
-  if (p.tail) pdl_wait();  // the window pass (previous launch) has finished every row
+  // PDL (every mode): the previous launch — the window pass or the batch kernel in tail / fallback
+  // mode, any kernel standalone — has finished and its writes are visible; the next launch may be
+  // scheduled while we run
+  pdl_wait();
+  pdl_trigger();
   unsigned long long t_start = 0;
   int n_rows = 0, n_passes = 0;
   if (p.timing && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
@@ -330,7 +334,7 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
   cfg.attrs = at;
-  cfg.numAttrs = tail ? 2 : 1;
+  cfg.numAttrs = 1;  // (the occupancy query below runs on the cluster shape alone; PDL added for the launch)
   cfg.gridDim = dim3((unsigned)pl.csize, 1, 1);
   int maxc = 0;
   if (!occ_cache_get((const void*)kern, pl.csize * 4 + (tail ? 1 : 0), &maxc)) {
@@ -342,6 +346,7 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   const int64_t ncl = std::min<int64_t>(a.batch, (int64_t)maxc);
   p.nclusters = (int)ncl;
   cfg.gridDim = dim3((unsigned)(ncl * pl.csize), 1, 1);
+  cfg.numAttrs = 2;
   if (!tail && a.events && a.n_events > 0) cudaEventRecord((cudaEvent_t)a.events[0], s);
   e = cudaLaunchKernelEx(&cfg, kern, p);
   if (!tail && a.events && a.n_events > 1) cudaEventRecord((cudaEvent_t)a.events[1], s);

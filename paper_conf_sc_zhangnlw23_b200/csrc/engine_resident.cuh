@@ -71,7 +71,7 @@ __device__ __forceinline__ void rstamp(const ResidentParams& p, int f) {
 
 template <typename W>
 struct ResShared {
-  unsigned hist[2][kMaxBins + 32];  // this CTA's histogram of the current pass (read remotely) + dummy bin
+  alignas(16) unsigned hist[2][kMaxBins + 32];  // this CTA's histogram of the current pass (read remotely) + dummy bin
   SelScratch<W, kRWarps> sel;
   unsigned long long tmp[kRWarps];
   ScanResult res;
@@ -89,6 +89,10 @@ __global__ void __launch_bounds__(kRBlock, 1) resident_kernel(const ResidentPara
   extern __shared__ __align__(16) unsigned char res_smem[];
   __shared__ ResShared<W> sh;
   cg::cluster_group cl = cg::this_cluster();
+  // PDL: launched while the previous kernel of the stream runs; nothing global is touched before
+  // its writes are visible. The next launch may then be scheduled (its launch latency overlaps us).
+  pdl_wait();
+  pdl_trigger();
   const int CS = (int)cl.num_blocks(), crank = (int)cl.block_rank();
   const int cid = blockIdx.x / CS;
   const int tid = threadIdx.x, lane = tid & 31;
@@ -200,14 +204,25 @@ __global__ void __launch_bounds__(kRBlock, 1) resident_kernel(const ResidentPara
       rstamp(p, 2 + 3 * min(q, 2));
       cl.sync();  // every CTA's histogram of digit q is complete
       rstamp(p, 3 + 3 * min(q, 2));
-      // sum the CS histograms bin-wise (DSMEM) and scan: the same j, K, C in every CTA
-      const ScanResult r = scan_choose<kRBlock>(
-          [&](int b) {
-            unsigned long long v = 0;
-            for (int rr = 0; rr < CS; ++rr) v += cl.map_shared_rank(hist, rr)[b];
-            return v;
-          },
-          1 << dh.width, K, sh.tmp, &sh.res);
+      // sum the CS histograms bin-wise (DSMEM) and scan: the same j, K, C in every CTA. Thread t
+      // owns bins 2t, 2t+1 (scan_choose's split): ONE 8-byte remote load per cluster rank, all CS
+      // loads in flight together (a rolled loop of 4-byte loads serialised ~16 DSMEM round trips)
+      static_assert((kMaxBins + kRBlock - 1) / kRBlock == 2, "two bins per thread");
+      unsigned s0 = 0, s1 = 0;
+      {
+        uint2 x[kMaxResCluster];
+#pragma unroll
+        for (int rr = 0; rr < kMaxResCluster; ++rr)
+          if (rr < CS) x[rr] = *(const uint2*)(cl.map_shared_rank(hist, rr) + 2 * tid);
+#pragma unroll
+        for (int rr = 0; rr < kMaxResCluster; ++rr)
+          if (rr < CS) {
+            s0 += x[rr].x;
+            s1 += x[rr].y;
+          }
+      }
+      const ScanResult r = scan_choose<kRBlock>([&](int b) { return (unsigned long long)((b & 1) ? s1 : s0); },
+                                                1 << dh.width, K, sh.tmp, &sh.res);
       rstamp(p, 4 + 3 * min(q, 2));
       K -= r.before;
       C = r.cnt;
@@ -311,11 +326,13 @@ cudaError_t launch_resident_kind(const SelectArgs& a, const Plan& pl, void* ws, 
   p.timing_n = a.trace ? a.batch * kTraceMaxPasses * kTraceFields : 0;
   p.vec_ok = ((uintptr_t)a.keys % 16 == 0) && ((size_t)a.len * sizeof(U)) % 16 == 0 ? 1 : 0;
   cudaLaunchConfig_t cfg = {};
-  cudaLaunchAttribute at[1];
+  cudaLaunchAttribute at[2];
   at[0].id = cudaLaunchAttributeClusterDimension;
   at[0].val.clusterDim.x = pl.csize;
   at[0].val.clusterDim.y = 1;
   at[0].val.clusterDim.z = 1;
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.blockDim = dim3(kRBlock);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
@@ -333,6 +350,7 @@ cudaError_t launch_resident_kind(const SelectArgs& a, const Plan& pl, void* ws, 
   p.nclusters = (int)std::min<int64_t>(a.batch, (int64_t)maxc);
   if (getenv("AIRTOPK_RES_ONECLUSTER")) p.nclusters = 1;  // debug: rows one after another (warm caches)
   cfg.gridDim = dim3((unsigned)(p.nclusters * pl.csize));
+  cfg.numAttrs = 2;  // + PDL (the occupancy query above ran on the cluster shape alone)
   if (a.events && a.n_events > 0) cudaEventRecord((cudaEvent_t)a.events[0], s);
   e = cudaLaunchKernelEx(&cfg, kern, p);
   if (a.events && a.n_events > 1) cudaEventRecord((cudaEvent_t)a.events[1], s);
