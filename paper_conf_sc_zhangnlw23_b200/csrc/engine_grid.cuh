@@ -85,6 +85,10 @@ constexpr int kGridBU = AIRTOPK_GRID_BU;  // buffer entries per thread per itera
 constexpr int kSmallFinish = 1024;  // max buffer entries of the single-CTA finish (shared memory)
 
 constexpr int kWarps = kBlock / 32;
+#ifndef AIRTOPK_WINDOW_L2PRE
+#define AIRTOPK_WINDOW_L2PRE 0
+#endif
+constexpr int kWindowL2Pre = AIRTOPK_WINDOW_L2PRE;  // chunks per CTA prefetched into L2 before the PDL wait
 
 #ifndef AIRTOPK_MINB
 #define AIRTOPK_MINB 2
@@ -134,10 +138,12 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   // writes) are requested BEFORE the PDL wait, so they stream in while the sample kernel finishes.
   // (The keys' producer completed before the sample kernel passed its own wait and triggered us.)
   int pre_issued = 0;
-  if constexpr (DF == 3 && TMA)
-    pre_issued = tma_prologue<typename KT<KIND>::U, HC, kBlock>((const typename KT<KIND>::U*)p.keys + row * p.len,
-                                                                p.len, cta, p.cpr, false,
+  if constexpr (DF == 3 && TMA) {
+    const typename KT<KIND>::U* rp = (const typename KT<KIND>::U*)p.keys + row * p.len;
+    pre_issued = tma_prologue<typename KT<KIND>::U, HC, kBlock>(rp, p.len, cta, p.cpr, false,
                                                                 smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>());
+    tma_prefetch_l2<typename KT<KIND>::U, kBlock>(rp, p.len, cta, p.cpr, tma_stages<HC>(), kWindowL2Pre);
+  }
   pdl_wait();     // the previous pass's scan (row state, buffers) is complete and visible
   pdl_trigger();  // the next pass may be scheduled as our CTAs retire (hides launch latency)
 

@@ -230,6 +230,28 @@ __device__ __forceinline__ int tma_prologue(const U* rowp, int64_t len, int slic
   return st;
 }
 
+// L2 prefetch (cp.async.bulk.prefetch.L2) of this CTA's chunks [from, from + count) of a forward TMA
+// pass (thread 0): the window pass issues it before its PDL wait, so HBM keeps streaming while the
+// sample kernel finishes (the ring alone holds only its first NST chunks).
+template <typename U, int BLOCK>
+__device__ __forceinline__ void tma_prefetch_l2(const U* rowp, int64_t len, int slice, int nslices, int from,
+                                                int count) {
+  constexpr int VEC = 16 / sizeof(U);
+  constexpr int NVT = (int)(kTmaChunk / 16 / BLOCK);
+  constexpr int64_t CV = (int64_t)BLOCK * NVT;
+  if (threadIdx.x != 0 || count <= 0) return;
+  const uintptr_t mis = (uintptr_t)rowp & 15u;
+  const int64_t head = mis ? std::min<int64_t>(len, (int64_t)((16u - mis) / sizeof(U))) : 0;
+  const int64_t nvec = (len - head) / VEC;
+  const uint4* vp = (const uint4*)(rowp + head);
+  const int64_t nch = nvec / CV;
+  const int64_t mine = (nch > slice) ? (nch - 1 - slice) / nslices + 1 : 0;
+  for (int64_t i = from; i < mine && i < (int64_t)from + count; ++i)
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(vp + ((int64_t)slice + i * nslices) * CV),
+                 "r"(kTmaChunk)
+                 : "memory");
+}
+
 // Runs the pass over this CTA's slice; the queues are flushed on return. Returns the number of
 // elements of the whole source (for the trace).
 template <int KIND, typename IdxT, int DF, int DH, bool HASIDX, int BLOCK, int HCOPIES = 0, bool TMA = false,
