@@ -137,6 +137,9 @@ typedef struct {
                            keys for select-min, descending for select-max; equal keys by ascending
                            index) — one extra launch, K <= 4096 (else AIRTOPK_EINVAL). 0 = unordered
                            (GridSelect rows are always sorted). */
+  int64_t trace_len;    /* int64 entries of `trace` (0 = the size stated there). The cluster, batched and
+                           resident engines write per-CTA debug timing stamps into `trace` instead of
+                           the per-row records; they never write past trace_len entries. */
 } airtopk_options;
 
 #define AIRTOPK_TRACE_MAX_PASSES 16

@@ -84,6 +84,7 @@ def _opts(alpha=0, engine=ENGINE_AUTO, ctas_per_row=0, cluster_size=0, trace=Non
         return o
     o = _build_opts(alpha, engine, ctas_per_row, cluster_size, window, tma, early_stop, sorted_out)
     o.trace = trace.data_ptr() if trace is not None else None
+    o.trace_len = trace.numel() if trace is not None else 0
     o.status = status.data_ptr() if status is not None else None
     if events is not None:
         # events: a ctypes array of cudaEvent_t handles (see make_event_array)

@@ -44,6 +44,7 @@ class Options(ctypes.Structure):
         ("early_stop", ctypes.c_int32),
         ("status", ctypes.c_void_p),
         ("sorted", ctypes.c_int32),
+        ("trace_len", ctypes.c_int64),
     ]
 
 

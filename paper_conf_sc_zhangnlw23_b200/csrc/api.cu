@@ -381,6 +381,7 @@ static SelectArgs make_args(const void* keys, int dt, int64_t batch, int64_t len
     a.ctas_per_row = opt->ctas_per_row;
     a.cluster_size = opt->cluster_size;
     a.trace = opt->trace;
+    a.trace_len = opt->trace_len;
     a.events = opt->events;
     a.n_events = opt->events ? opt->n_events : 0;
     a.window = opt->window;

@@ -27,6 +27,7 @@ struct SelectArgs {
   unsigned* status = nullptr;       // optional device word: row error flags OR-ed in after the select
   int sorted = 0;                   // 1: rows sorted in selection order after the select (K <= 4096)
   int64_t* trace = nullptr;
+  int64_t trace_len = 0;  // int64 entries of trace (0: batch * kTraceMaxPasses * kTraceFields)
   void* const* events = nullptr;    // optional cudaEvent_t[n_events] recorded around launches
   int n_events = 0;
 };

@@ -702,7 +702,7 @@ cudaError_t launch_batch_kind(const SelectArgs& a, const Plan& pl, void* ws, cud
   p.nsamp = pl.nsamp;
   p.early_stop = a.early_stop;
   p.timing = a.trace;
-  p.timing_n = a.batch * kTraceMaxPasses * kTraceFields;
+  p.timing_n = a.trace_len > 0 ? a.trace_len : a.batch * kTraceMaxPasses * kTraceFields;
   const int G = num_sms() * std::min(occ, 1);
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)G);

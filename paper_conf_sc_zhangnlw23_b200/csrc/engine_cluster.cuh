@@ -344,6 +344,12 @@ cudaError_t launch_cluster_t(const SelectArgs& a, const Plan& pl, void* ws, cuda
   }
   if (maxc < 1) return cudaErrorInvalidConfiguration;
   const int64_t ncl = std::min<int64_t>(a.batch, (int64_t)maxc);
+  // the per-CTA timing must fit the caller's trace buffer (batch x kTraceMaxPasses x kTraceFields
+  // int64 or trace_len, airtopk.h): otherwise no timing (debug only) — never an out-of-bounds write
+  //
+  if (p.timing && ncl * pl.csize * (int64_t)p.timing_stride >
+                      (a.trace_len > 0 ? a.trace_len : a.batch * kTraceMaxPasses * kTraceFields))
+    p.timing = nullptr;
   p.nclusters = (int)ncl;
   cfg.gridDim = dim3((unsigned)(ncl * pl.csize), 1, 1);
   cfg.numAttrs = 2;

@@ -323,7 +323,7 @@ cudaError_t launch_resident_kind(const SelectArgs& a, const Plan& pl, void* ws, 
   p.slice = pl.rslice;
   p.early_stop = a.early_stop;
   p.timing = a.trace;
-  p.timing_n = a.trace ? a.batch * kTraceMaxPasses * kTraceFields : 0;
+  p.timing_n = a.trace ? (a.trace_len > 0 ? a.trace_len : a.batch * kTraceMaxPasses * kTraceFields) : 0;
   p.vec_ok = ((uintptr_t)a.keys % 16 == 0) && ((size_t)a.len * sizeof(U)) % 16 == 0 ? 1 : 0;
   cudaLaunchConfig_t cfg = {};
   cudaLaunchAttribute at[2];
