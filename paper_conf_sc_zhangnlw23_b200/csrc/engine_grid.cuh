@@ -89,6 +89,10 @@ constexpr int kWarps = kBlock / 32;
 #define AIRTOPK_WINDOW_L2PRE 0
 #endif
 constexpr int kWindowL2Pre = AIRTOPK_WINDOW_L2PRE;  // chunks per CTA prefetched into L2 before the PDL wait
+#ifndef AIRTOPK_WINDOW_EARLY
+#define AIRTOPK_WINDOW_EARLY 1
+#endif
+constexpr bool kWindowEarly = AIRTOPK_WINDOW_EARLY != 0;  // window pass: ring stages issued before the PDL wait
 
 #ifndef AIRTOPK_MINB
 #define AIRTOPK_MINB 2
@@ -138,7 +142,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   // writes) are requested BEFORE the PDL wait, so they stream in while the sample kernel finishes.
   // (The keys' producer completed before the sample kernel passed its own wait and triggered us.)
   int pre_issued = 0;
-  if constexpr (DF == 3 && TMA) {
+  if constexpr (DF == 3 && TMA && kWindowEarly) {
     const typename KT<KIND>::U* rp = (const typename KT<KIND>::U*)p.keys + row * p.len;
     pre_issued = tma_prologue<typename KT<KIND>::U, HC, kBlock>(rp, p.len, cta, p.cpr, false,
                                                                 smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>());
@@ -218,7 +222,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   c.err = &st->error;
   c.hist = sh_hist;
   c.ring = smem_addr(sh_hist) + (unsigned)tma_ring_offset<HC>();
-  c.pre = (DF == 3 && TMA);
+  c.pre = (DF == 3 && TMA && kWindowEarly);
   c.wq = &sh_wq[HAS_Q ? warp : 0];
 
   if constexpr (FILTER && DH != 0) {

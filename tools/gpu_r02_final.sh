@@ -30,9 +30,9 @@ timeout 300 ncu --metrics $M --clock-control none -c 40 --csv --log-file $O/laun
 timeout 300 ncu --metrics $M --clock-control none -c 60 --csv --log-file $O/launches_split_step.csv \
   python tools/split_step.py > $O/split_step.log 2>&1
 # full captures of the dominant kernels
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:pass_kernel -s 2 -c 1 -o $O/full_c3_window python tools/prof_select.py --config c3 --reps 2 > $O/ncu_c3.log 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:pass_kernel -s 2 -c 1 -o $O/full_c3_window python tools/prof_select.py --config c3 --reps 3 > $O/ncu_c3.log 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:batch_kernel -s 1 -c 1 -o $O/full_c2_batch python tools/prof_select.py --config c2 --reps 2 > $O/ncu_c2.log 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:pass_kernel -s 2 -c 1 -o $O/full_c4_window python tools/prof_select.py --config c4 --reps 2 > $O/ncu_c4.log 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:pass_kernel -s 2 -c 1 -o $O/full_c4_window python tools/prof_select.py --config c4 --reps 3 > $O/ncu_c4.log 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:tail_kernel -s 1 -c 1 -o $O/full_c3_tail python tools/prof_select.py --config c3 --reps 2 > $O/ncu_c3t.log 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:resident_kernel -s 1 -c 1 -o $O/full_c1_resident python tools/prof_select.py --config c1 --reps 2 > $O/ncu_c1.log 2>&1
 for r in 100 50 25 13; do python tools/batch_timing.py $r >> $O/batch_timing.txt 2>/dev/null; done
