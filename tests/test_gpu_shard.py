@@ -122,6 +122,25 @@ def test_out_and_workspace_checks():
         at.select(x, 10, workspace=torch.empty(1 << 20, dtype=torch.float32, device="cuda"))
 
 
+@pytest.mark.parametrize("engine,shape,k", [(2, (1, 1 << 17), 32), (5, (8, 1 << 18), 64), (6, (1, 1 << 16), 32)])
+def test_debug_timing_bounded_by_trace_len(engine, shape, k):
+    """Engines that write per-CTA debug stamps into the trace buffer never write past the buffer the
+    caller passed (options.trace_len; the cluster engine's stamps could overrun it)."""
+    import torch
+    import paper_conf_sc_zhangnlw23_b200 as at
+    x = torch.from_numpy(gen.uniform_f32(41, shape[0] * shape[1]).reshape(shape)).cuda()
+    kw = {"cluster_size": 16} if engine == 2 else {}
+    big = torch.zeros(1 << 16, dtype=torch.int64, device="cuda")
+    at.select(x, k, engine=engine, trace=big[:24], **kw)
+    torch.cuda.synchronize()
+    assert int(torch.count_nonzero(big[24:]).item()) == 0
+    v, i = at.select(x, k, engine=engine, trace=big, **kw)
+    torch.cuda.synchronize()
+    assert int(torch.count_nonzero(big).item()) > 0   # stamps are written when they fit
+    rv, ri = oracle.topk_nth(x.cpu().numpy(), k)
+    assert np.array_equal(np.sort(i.cpu().numpy(), axis=1), np.sort(ri, axis=1))
+
+
 def test_select_on_non_current_device():
     import torch
     import paper_conf_sc_zhangnlw23_b200 as at
