@@ -54,7 +54,10 @@ constexpr unsigned kBStage = kBatchStage;     // bytes per bulk-copy ring stage 
 #ifndef AIRTOPK_BATCH_STAGES
 #define AIRTOPK_BATCH_STAGES 8
 #endif
-constexpr int kBStages = AIRTOPK_BATCH_STAGES;  // ring depth: 8 x 24 KiB = 192 KiB in flight per SM
+constexpr int kBStages = AIRTOPK_BATCH_STAGES;
+#ifndef AIRTOPK_BATCH_PDL
+#define AIRTOPK_BATCH_PDL 0  // measured: no gain on c2 (the fallback launch already overlaps); off
+#endif  // ring depth: 8 x 24 KiB = 192 KiB in flight per SM
 constexpr int kBPre = 4;                      // stages issued before the sampling phase
 #ifndef AIRTOPK_BATCH_L2PRE
 #define AIRTOPK_BATCH_L2PRE 0  // measured: L2 prefetches during phase A slow the sampling, stream unchanged
@@ -542,6 +545,12 @@ __global__ void __launch_bounds__(kBBlock, 1) batch_kernel(const BatchParams p) 
   const unsigned fullb = ring + (unsigned)kBRingBytes, emptyb = fullb + 8u * kBStages;
   const int64_t nch = p.batch * (int64_t)p.cpc;
   const int64_t mine = cta < nch ? (nch - 1 - cta) / G + 1 : 0;  // chunks cta, cta + G, ...
+#if AIRTOPK_BATCH_PDL
+  // PDL: launched while the previous kernel of the stream (e.g. the previous select's fallback
+  // launch) runs; nothing global is touched before its writes are visible
+  pdl_wait();
+  pdl_trigger();
+#endif
   bstamp(p, 0);
   // the first kBPre chunks this CTA streams start landing in the ring while the rows are sampled
   if (tid < kBStages) sh_scnt[tid] = 0;
@@ -709,11 +718,13 @@ cudaError_t launch_batch_kind(const SelectArgs& a, const Plan& pl, void* ws, cud
   cfg.blockDim = dim3(kBBlock);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
-  cudaLaunchAttribute at[1];
+  cudaLaunchAttribute at[2];
   at[0].id = cudaLaunchAttributeCooperative;
   at[0].val.cooperative = 1;
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = AIRTOPK_BATCH_PDL ? 2 : 1;
   if (a.events && a.n_events > 0) cudaEventRecord((cudaEvent_t)a.events[0], s);
   e = cudaLaunchKernelEx(&cfg, kern, p);
   if (e != cudaSuccess) return e;

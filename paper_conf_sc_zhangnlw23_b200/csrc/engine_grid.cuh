@@ -984,7 +984,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocksFilter) tail_kernel(const Gr
   __shared__ WarpQ<U, IdxT> sh_wq[kWarps];
   __shared__ unsigned long long sh_tmp[kWarps];
   __shared__ ScanResult sh_res;
-  pdl_wait();  // the window pass (previous launch) is complete
+  pdl_wait();     // the window pass (previous launch) is complete
+  pdl_trigger();  // the next select's first launch may be scheduled (it waits for our completion)
   const RowState* st = p.st;
   TailState S;
   int q;
