@@ -85,6 +85,16 @@ constexpr int kGridBU = AIRTOPK_GRID_BU;  // buffer entries per thread per itera
 constexpr int kSmallFinish = 1024;  // max buffer entries of the single-CTA finish (shared memory)
 
 constexpr int kWarps = kBlock / 32;
+#ifndef AIRTOPK_TMA_FILTER_HC
+#define AIRTOPK_TMA_FILTER_HC 2  // measured (c3, paper passes): pass 2 741 -> 722 us (6 instead of 5 ring stages); c4 unchanged
+#endif
+// Histogram copies of a grid pass. Bulk-copy (TMA) filter passes may use fewer copies than the
+// register path (AIRTOPK_TMA_FILTER_HC > 0): the shared memory saved becomes ring stages.
+template <int KIND, typename IdxT, int DF, bool TMA>
+__host__ __device__ constexpr int pass_hc() {
+  return (TMA && (DF == 1 || DF == 2) && AIRTOPK_TMA_FILTER_HC > 0) ? AIRTOPK_TMA_FILTER_HC
+                                                                      : hist_copies<KIND, IdxT, DF>();
+}
 #ifndef AIRTOPK_WINDOW_L2PRE
 #define AIRTOPK_WINDOW_L2PRE 0
 #endif
@@ -125,7 +135,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
   using CountT = std::conditional_t<sizeof(IdxT) == 8, unsigned long long, unsigned>;
   constexpr bool HAS_Q = DF != 0;
   constexpr bool FILTER = (DF == 1 || DF == 2);  // Alg1 L15-22 filter of digit q-1
-  constexpr int HC = hist_copies<KIND, IdxT, DF>();
+  constexpr int HC = pass_hc<KIND, IdxT, DF, TMA>();
 
   extern __shared__ unsigned sh_hist[];  // kHistSlots * HC counters (dynamic: may exceed 48 KB)
   __shared__ WarpQ<U, IdxT> sh_wq[HAS_Q ? kWarps : 1];  // per-warp tagged result / candidate queues
@@ -243,7 +253,7 @@ __global__ void __launch_bounds__(kBlock, TMA ? 1 : (DF == 0 ? kMinBlocks : kMin
     __syncthreads();
   }
 
-  const unsigned long long nread = run_pass<KIND, IdxT, DF, DH, HASIDX, kBlock, 0, TMA, kGridBU>(c);
+  const unsigned long long nread = run_pass<KIND, IdxT, DF, DH, HASIDX, kBlock, HC, TMA, kGridBU>(c);
   dbg_stamp(p.trace, row, q, 1, 1, p.P);
   if (cta == 0) dbg_stamp(p.trace, row, q, 5, 2, p.P);
 
@@ -606,7 +616,10 @@ __global__ void __launch_bounds__(kSampleBlock) sample_kernel(const GridParams p
   // stratified positions: a DRAM line is fetched whole anyway, so this costs nsamp*4 bytes of traffic
   // instead of nsamp*128. (Runs are independent draws for i.i.d. data; a row whose order defeats the
   // estimate only triggers the fallback.)
-  constexpr int kRun = 32;
+#ifndef AIRTOPK_SAMPLE_RUN
+#define AIRTOPK_SAMPLE_RUN 32
+#endif
+  constexpr int kRun = AIRTOPK_SAMPLE_RUN;  // (A/B: longer runs touch fewer pages of a long row)
   const int nruns = nsamp / kRun;
   const int64_t stride = p.len / nruns;
   // phase 1: this CTA's runs part, part + cps, ... (all loads in flight at once)
@@ -760,9 +773,9 @@ struct Events {
 
 template <int KIND, typename IdxT, int DF, int DH, bool TMA = false>
 constexpr size_t hist_smem_bytes() {
-  static_assert(!(DF == 1 || DF == 2) || DH == 0 || (size_t)kHistSlots * 4 * hist_copies<KIND, IdxT, DF>() >=
+  static_assert(!(DF == 1 || DF == 2) || DH == 0 || (size_t)kHistSlots * 4 * pass_hc<KIND, IdxT, DF, TMA>() >=
                     (size_t)kSmallFinish * (sizeof(typename KT<KIND>::U) + sizeof(IdxT)), "small finish smem");
-  constexpr int HC = hist_copies<KIND, IdxT, DF>();
+  constexpr int HC = pass_hc<KIND, IdxT, DF, TMA>();
   return TMA ? tma_smem_bytes<HC>() : (size_t)kHistSlots * 4 * HC;
 }
 
