@@ -103,6 +103,10 @@ constexpr int kWindowL2Pre = AIRTOPK_WINDOW_L2PRE;  // chunks per CTA prefetched
 #define AIRTOPK_WINDOW_EARLY 1
 #endif
 constexpr bool kWindowEarly = AIRTOPK_WINDOW_EARLY != 0;  // window pass: ring stages issued before the PDL wait
+#ifndef AIRTOPK_TAIL_IDENT
+#define AIRTOPK_TAIL_IDENT 1
+#endif
+constexpr bool kTailIdent = AIRTOPK_TAIL_IDENT != 0;  // fused tail: identity-filter elision
 
 #ifndef AIRTOPK_MINB
 #define AIRTOPK_MINB 2
@@ -870,6 +874,8 @@ struct TailState {
   unsigned long long K, C, tcode, tidx, nbuf;
   int src1;   // 0 = input row L, s + 1 = candidate buffer slot s
   int stop1;  // 1 + digit after whose scan K == C (early stop); 0 = none
+  int ident;  // the last scan put every candidate into the target bin (C unchanged): the next filter
+              // is the identity, so a buffer-source pass only histograms its next digit (no copy)
 };
 
 template <int KIND, typename IdxT, int DF, int DH>
@@ -886,7 +892,9 @@ __device__ __forceinline__ bool tail_pass(const GridParams& p, int q, TailState&
   c.q = q;
   c.emit_all = FILTER && ((S.stop1 != 0 && S.stop1 - 1 == q - 1) || DH == 0);
   c.do_hist = (DH != 0) && !c.emit_all;
-  const unsigned long long Cin = FILTER ? S.C : (unsigned long long)p.len;
+  // DF == 0 over a candidate buffer: identity-filter elision (S.ident) — histogram digit q of the
+  // buffer as it stands; nothing is emitted or stored
+  const unsigned long long Cin = (FILTER || S.src1 > 0) ? S.C : (unsigned long long)p.len;
   c.srcL = (S.src1 == 0);
   c.store = c.do_hist && FILTER && (Cin <= (unsigned long long)p.cap_rule);  // Alg1 L17
   c.sel_min = p.sel_min != 0;
@@ -923,6 +931,7 @@ __device__ __forceinline__ bool tail_pass(const GridParams& p, int q, TailState&
   c.hist = sh_hist;
   c.ring = 0;
   c.wq = &wq[tid >> 5];
+  c.dbg = (p.tstamp && q < 16) ? p.tstamp + 64 + q * 4 : nullptr;  // debug: run_pass internals
   if constexpr (FILTER && DH != 0) {
     // small finish: one CTA ends the row; the decision is grid-uniform
     if (!c.emit_all && !c.srcL && c.nbuf <= (unsigned long long)p.small_finish) {
@@ -968,8 +977,9 @@ __device__ __forceinline__ bool tail_pass(const GridParams& p, int q, TailState&
   const unsigned long long newK = S.K - r.before, newC = r.cnt;  // Alg1 L26-28
   if (c.store) {
     S.src1 = sslot + 1;
-    S.nbuf = __ldcg(c.bufc);
+    S.nbuf = Cin;  // every candidate of the filter was stored: hist[j] of the previous scan (no L2 read)
   }
+  S.ident = (newC == Cin) ? 1 : 0;
   S.C = newC;
   S.K = newK;
   if (!c.dh.is_idx) S.tcode |= (unsigned long long)r.j << c.dh.shift;
@@ -1011,6 +1021,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocksFilter) tail_kernel(const Gr
     S.src1 = st->src1;
     S.stop1 = st->stop1;
     S.nbuf = S.src1 > 0 ? st->buf_count[S.src1 - 1] : 0ull;
+    S.ident = (st->C == st->Cp) ? 1 : 0;  // the window scan kept every member (e.g. c4: digit 1 is one bin)
   } else {  // no window / the window missed: the paper's passes from L
     q = 0;
     S.K = (unsigned long long)p.k;
@@ -1019,6 +1030,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocksFilter) tail_kernel(const Gr
     S.src1 = 0;
     S.stop1 = 0;
     S.nbuf = 0;
+    S.ident = 0;
   }
 #pragma unroll 1
   for (; q <= p.P; ++q) {
@@ -1026,7 +1038,11 @@ __global__ void __launch_bounds__(kBlock, kMinBlocksFilter) tail_kernel(const Gr
     const int DF = q == 0 ? 0 : (digit_of(q - 1, KT<KIND>::R, p.IB).is_idx ? 2 : 1);
     const int DH = q == p.P ? 0 : (digit_of(q, KT<KIND>::R, p.IB).is_idx ? 2 : 1);
     bool done;
-    switch (DF * 3 + DH) {
+    // identity-filter elision: after a scan that kept every candidate (S.ident), a pass over a buffer
+    // that would filter a key digit and histogram the next key digit only histograms (no emit, no copy)
+    const bool ident = kTailIdent && S.ident && S.src1 > 0 && DF == 1 && DH == 1 &&
+                       !(S.stop1 != 0 && S.stop1 - 1 == q - 1);
+    switch (ident ? 0 * 3 + 1 : DF * 3 + DH) {
       case 0 * 3 + 1: done = tail_pass<KIND, IdxT, 0, 1>(p, q, S, sh_hist, sh_wq, sh_tmp, &sh_res); break;
       case 1 * 3 + 1: done = tail_pass<KIND, IdxT, 1, 1>(p, q, S, sh_hist, sh_wq, sh_tmp, &sh_res); break;
       case 1 * 3 + 2: done = tail_pass<KIND, IdxT, 1, 2>(p, q, S, sh_hist, sh_wq, sh_tmp, &sh_res); break;

@@ -194,7 +194,16 @@ struct PassCtx {
   unsigned* hist;  // shared, kMaxBins * hist_copies() counters, zeroed by the caller
   unsigned ring;   // TMA streaming: shared-window address of the ring (after the histogram copies)
   WarpQ<U, IdxT>* wq;
+  int64_t* dbg = nullptr;  // debug (fused tail stamps): CTA 0's %globaltimer at points of the pass
 };
+
+__device__ __forceinline__ void pass_dbg(int64_t* d, int i) {
+  if (d != nullptr && blockIdx.x == 0 && threadIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    d[i] = (int64_t)t;
+  }
+}
 
 // First stages of the bulk-copy ring of a TMA pass over the input row (thread 0: barrier init + up to
 // NST copies). Returns the number of stages issued (thread 0).
@@ -721,9 +730,11 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
           hist_cand(code[j], idx[j], cand);
           push1(win || (cand && store), win ? 0 : 1, code[j], idx[j]);
         }
+        pass_dbg(c.dbg, 0);
       }
     }
   }
+  pass_dbg(c.dbg, 1);
   if constexpr (DF != 0) {
     // final flush of the partial queues, aggregated over the CTA: one global atomic per CTA and
     // destination instead of one per warp (same-address atomics serialise in L2: ~1 per ns)
@@ -754,9 +765,11 @@ __device__ __forceinline__ unsigned long long run_pass(const PassCtx<typename KT
       }
     }
     __syncthreads();
+    pass_dbg(c.dbg, 2);
     if (qcnt)
       wq_write<KIND, IdxT>(wq, qcnt, s_base[0][warp], s_base[1][warp], c.ov, c.oi, c.kk, c.bco, c.bio, c.capa,
                            sel_min, c.err, c.ioff);
+    pass_dbg(c.dbg, 3);
   }
   if constexpr (DF == 3) {  // one atomic per warp: window-member extremes (the tail skips digits
                             // on which all members agree)

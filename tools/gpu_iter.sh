@@ -1,8 +1,7 @@
 #!/bin/bash
-# A/B: histogram copies of the bulk-copy filter passes (paper path: --window -1), c3 / c4 / c3-adversarial-like
+# iteration: GPU tests + fuzz, fused-tail stamps, c3/c4 A/B vs a variant library
 O=gpurun_out/iter; rm -rf $O; mkdir -p $O
-for l in paper_conf_sc_zhangnlw23_b200/libairtopk.so build_var/lib_hc2.so; do
-  echo "== $l" >> $O/probe.txt
-  for c in c3 c4; do AIRTOPK_LIB=$l timeout 200 python tools/probe_select.py --config $c --window -1 >> $O/probe.txt 2>&1; done
-  AIRTOPK_LIB=$l timeout 600 python -m pytest tests/test_gpu_parity.py -q -x -k "tma or paper or trace" 2>&1 | tail -1 >> $O/probe.txt
-done
+timeout 1200 python -m pytest tests -m gpu -q -x 2>&1 | tail -4 > $O/pytest.log
+timeout 200 python tests/fuzz_gpu.py 150 91 > $O/fuzz.txt 2>&1
+for a in "28 50000 adversarial" "30 1048576 uniform"; do AIRTOPK_TAIL_STAMPS=1 timeout 120 python tools/tail_stamps.py $a >> $O/tail_stamps.txt 2>&1; done
+CONFIGS="c3 c4" bash tools/gpu_libab2.sh build_var/lib_noident.so
