@@ -22,6 +22,9 @@ struct SelScratch {
   unsigned long long tmp[NW];
   ScanResult res;
   W wmin[NW], wmax[NW];
+  W cw[32];          // <= 32 live entries compacted for warp 0's rank count
+  unsigned ci[32];
+  unsigned cn;
 };
 
 // Entry e = tid + t * BLOCK (t < tcnt, block-uniform) is live iff bit t of `valid`. C = number of
@@ -44,12 +47,15 @@ __device__ void block_select_smem(const typename KT<KIND>::U* stc, const unsigne
       const bool v = valid & 1u;
       const U c = v ? stc[tid] : (U)0;
       const unsigned ix = v ? sti[tid] : 0u;
+      // rank by counting over the live lanes' entries, read as shared-memory broadcasts (independent
+      // loads: no serial shuffle chain)
+      const unsigned vm = __ballot_sync(kFull, v);
       unsigned rank = 0;
+#pragma unroll 8
       for (int o = 0; o < 32; ++o) {
-        const bool vo = __shfl_sync(kFull, (int)v, o);
-        const W co = (W)shfl((W)c, o);
-        const unsigned io = __shfl_sync(kFull, ix, o);
-        rank += vo && (co < (W)c || (co == (W)c && io < ix));
+        const W co = (W)stc[o];
+        const unsigned io = sti[o];
+        rank += ((vm >> o) & 1u) && (co < (W)c || (co == (W)c && io < ix));
       }
       emit(v && rank < Kr, c, ix);
     }
@@ -116,6 +122,35 @@ __device__ void block_select_smem(const typename KT<KIND>::U* stc, const unsigne
     Kr -= r.before;
     C = r.cnt;
     pos -= w;
+    if (C <= 32 && pos > 0 && !(Kr == C && early_stop)) {
+      // at most 32 live entries left: compact them into shared memory and let warp 0 rank them by
+      // counting (one shuffle round) instead of running the remaining histogram passes
+      if (tid == 0) sh.cn = 0;
+      __syncthreads();
+#pragma unroll 1
+      for (int t = 0, e = tid; t < tcnt; ++t, e += BLOCK) {
+        if ((valid >> t) & 1u) {
+          const unsigned slot = atomicAdd(&sh.cn, 1u);
+          sh.cw[slot] = (W)stc[e];
+          sh.ci[slot] = sti[e];
+        }
+      }
+      __syncthreads();
+      if (warp == 0) {
+        const bool v = lane < (int)C;
+        const W c = v ? sh.cw[lane] : (W)0;
+        const unsigned ix = v ? sh.ci[lane] : 0u;
+        unsigned rank = 0;
+#pragma unroll 8
+        for (int o = 0; o < 32; ++o) {
+          const W co = sh.cw[o];
+          const unsigned io = sh.ci[o];
+          rank += (o < (int)C) && (co < c || (co == c && io < ix));
+        }
+        emit(v && rank < Kr, (U)c, ix);
+      }
+      return;
+    }
   }
   // early stop (K == C) or the last digit: every remaining candidate is a result
 #pragma unroll 1
