@@ -131,7 +131,8 @@ def describe(dtype, batch: int, length: int, k: int, alpha: int = 0, engine: int
 def _stream(stream, device):
     torch = _torch()
     if stream is None:  # the raw cudaStream_t of torch's current stream (no Stream object built)
-        return torch._C._cuda_getCurrentRawStream(device.index)
+        raw = getattr(torch._C, "_cuda_getCurrentRawStream", None)
+        return raw(device.index) if raw is not None else torch.cuda.current_stream(device).cuda_stream
     if stream.device != device:
         raise ValueError(f"stream of {stream.device} used with tensors on {device}")
     return stream.cuda_stream
