@@ -106,6 +106,15 @@ int grid_vec_chunk(int kind);
 
 // Workspace layout (all offsets 256-aligned):
 //   [RowState x batch][2 histograms x 2048 counters x batch][code buffers 2 x batch x cap][index buffers]
+// batched engine: samples per row = len / div (clamped to 4K..16K); env AIRTOPK_BATCH_SAMP_DIV: A/B knob
+static int64_t batch_samp_div() {
+  static const int64_t d = [] {
+    const char* e = getenv("AIRTOPK_BATCH_SAMP_DIV");
+    return (e && atoll(e) > 0) ? (int64_t)atoll(e) : (int64_t)128;
+  }();
+  return d;
+}
+
 Plan make_plan(const SelectArgs& a) {
   Plan p{};
   p.R = key_bits(a.kind);
@@ -155,7 +164,7 @@ Plan make_plan(const SelectArgs& a) {
   if (!a.in_idx && a.window >= 0 && (a.engine == 0 || a.engine == 5) && a.len >= (int64_t(1) << 14) &&
       a.len < (int64_t(1) << 31)) {
     const int es = key_bytes(a.kind), vec = 16 / es;
-    int64_t ns = std::min<int64_t>(std::max<int64_t>(a.len / 128, 4096), 16384);
+    int64_t ns = std::min<int64_t>(std::max<int64_t>(a.len / batch_samp_div(), 4096), 16384);
     ns = std::min<int64_t>(ns, a.len / 2) / 32 * 32;
     if (es == 8) ns = std::min<int64_t>(ns, 8192);
     const double f = (double)a.k / (double)a.len, r = f * (double)ns;

@@ -1,12 +1,9 @@
 #!/bin/bash
-# iteration: batched / resident tests + fuzz, c2 stamps, c1/c2 A/B vs the previous library
+# A/B: samples per row of the batched engine (len/128 = 8K for c2 vs len/256 = 4K)
 O=gpurun_out/iter; rm -rf $O; mkdir -p $O
-timeout 1200 python -m pytest tests -m gpu -q -x 2>&1 | tail -4 > $O/pytest.log
-timeout 200 python tests/fuzz_gpu.py 150 97 > $O/fuzz.txt 2>&1
-for l in paper_conf_sc_zhangnlw23_b200/libairtopk.so build_var/lib_prev.so; do
-  echo "== $l" >> $O/batch_timing.txt
-  AIRTOPK_LIB=$l timeout 120 python tools/batch_timing.py 100 >> $O/batch_timing.txt 2>&1
-  AIRTOPK_LIB=$l timeout 120 python tools/resident_timing.py 65536 32 0 >> $O/batch_timing.txt 2>&1
+for d in 128 256; do
+  echo "== AIRTOPK_BATCH_SAMP_DIV=$d" >> $O/ab.txt
+  AIRTOPK_BATCH_SAMP_DIV=$d timeout 120 python tools/batch_timing.py 100 2>&1 | grep -v "Warn\|rel =\|med =\|slow CTA" >> $O/ab.txt
+  for rep in 1 2; do AIRTOPK_BATCH_SAMP_DIV=$d timeout 300 python bench.py --config c2 --no-cpu --no-extras --e2e-steps 1 2>/dev/null | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('c2', d['ms_per_step']*1e3, d['roofline']['frac'])" >> $O/ab.txt; done
+  AIRTOPK_BATCH_SAMP_DIV=$d timeout 600 python -m pytest tests/test_gpu_batch.py -q -x 2>&1 | tail -1 >> $O/ab.txt
 done
-rm -rf gpurun_out/ab2
-CONFIGS="c1 c2" bash tools/gpu_libab2.sh build_var/lib_prev.so
